@@ -1,0 +1,420 @@
+#!/usr/bin/env python
+"""bench.py — SYnergy fused predict+select on B200: kernel x frequency evaluations/s.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (one process per GPU, NCCL)
+
+A step = one pass of the whole hot path over one batch: synergy_sweep (model inference for
+every (kernel, clock) pair, default-clock normalisation, per-target objectives, masked argmin;
+PAPER §6.2) on the rank's kernels, then (N > 1) the NCCL all-gather that assembles
+the choice table.  Default workload = BASELINE.json configs[1] (c2: 1000 kernels x 196 clocks,
+100-tree depth-12 forests for speedup and energy, 6 targets) per rank, weak scaling (rank r
+sweeps its own 1000 kernels of the seeded population).  Inputs are resident in HBM; L2 is
+flushed (512 MiB write) between timed steps because the 13 MB model would otherwise stay in L2.
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "kernel x frequency evaluations/sec (fused predict+select)"
+UNIT = "evals/s"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--warmup", type=int, default=10)
+    p.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--flush-mib", type=int, default=512)
+    return p.parse_args()
+
+
+def dist_env():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)),
+            int(os.environ.get("LOCAL_RANK", 0)))
+
+
+def workload_desc(cfg):
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    n_k, n_f, sp, en, tg = W.CONFIGS[cfg]
+    m = lambda s: "linear" if s[0] == "lin" else f"RF {s[1]}xD{s[2]}"
+    tgt = "MAX_PERF,MIN_ENERGY,MIN_EDP,MIN_ED2P,ES_50,PL_50" if tg == "six" else "ES_25,ES_50,ES_75,PL_25,PL_50,PL_75"
+    return (f"{cfg}: {n_k} kernels x {n_f} core clocks, speedup {m(sp)}, energy {m(en)}, 12 static "
+            f"features, targets {tgt}")
+
+
+def decisions_per_eval(spec):
+    """Internal-node decisions per evaluation of one model (T*D for the complete trees the bench
+    configs use; the oracle counts the same quantity)."""
+    if spec.forest_weight == 0.0:
+        return 0
+    import numpy as np
+    # depth of each complete BFS tree: nodes = 2^(D+1)-1
+    sizes = np.diff(spec.tree_offset)
+    return int(sum(int(np.log2(int(s) + 1)) - 1 for s in sizes))
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def ncu_traffic(cfg):
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            return json.load(f).get(cfg, {}).get("k_sweep_dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------------- clock sampler
+
+class ClockSampler:
+    """NVML sampling of SM clock and clocks-event reasons during the timed region."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device_index, period_s=0.002):
+        self.samples, self.reasons_seen = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self.period = period_s
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            idx = int(vis.split(",")[device_index]) if vis else device_index
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.nv = pynvml
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.h = None
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                mhz = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+                rs = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.samples.append((mhz, rs))
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.h is not None:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.h is not None:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"], "samples": 0}
+        load = [(m, r) for m, r in self.samples if not (r & 0x1)] or self.samples
+        reasons = set()
+        for _, r in load:
+            for bit, name in self.REASONS.items():
+                if r & bit and bit != 0x1:
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(m for m, _ in load), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(reasons), "samples": len(self.samples), "samples_under_load": len(load)}
+
+
+# -------------------------------------------------------------------------- CPU oracle
+
+def _oracle_range(args):
+    cfg, row0, n, models_key = args
+    import oracle
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    w = _POOL_CACHE.get(models_key)
+    feats = W.make_features(cfg, row0, n)
+    t = time.perf_counter()
+    oracle.sweep(w[0], w[1], feats, w[2], w[3], w[4])
+    return time.perf_counter() - t
+
+
+_POOL_CACHE = {}
+
+
+def _pool_init(cfg):
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    import oracle
+    oracle.build()
+    sp, en, freqs, d = W.make_models(cfg)
+    tg = W.targets_six() if W.CONFIGS[cfg][4] == "six" else W.targets_es_pl()
+    _POOL_CACHE[cfg] = (sp, en, freqs, d, tg)
+
+
+def oracle_single_core(cfg, n_k_cap, budget_s=10.0):
+    """The oracle as it stands, one core, on the first kernels of the workload until ~budget_s."""
+    import oracle
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    oracle.build()
+    w = W.make_config(cfg, row0=0, n=min(n_k_cap, W.CONFIGS[cfg][0]))
+    evals = 0
+    t0 = time.perf_counter()
+    chunk = max(1, min(w.n_kernels, 100))
+    row = 0
+    passes = 0
+    while True:
+        r = oracle.sweep(w.speedup, w.energy, w.features[row:row + chunk], w.freqs, w.default_idx, w.targets)
+        evals += r["choice"].shape[0] * w.n_freqs
+        row += chunk
+        if row >= w.n_kernels:
+            row = 0
+            passes += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s and (passes >= 1 or el >= 3 * budget_s):
+            break
+    return evals / el, evals, el
+
+
+def run_reference(args, rank, world):
+    """Reference arm: the CPU oracle (as it stands, single-threaded per process) on the box's host
+    cores, one process per core over contiguous kernel ranges of a bounded sample per step."""
+    if rank != 0:
+        return
+    import multiprocessing as mp
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    cfg = args.config
+    n_k, n_f = W.CONFIGS[cfg][0], W.CONFIGS[cfg][1]
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+    sp, en, freqs, d = W.make_models(cfg)
+    dec = decisions_per_eval(sp) + decisions_per_eval(en)
+    # bounded sample: ~2 s of wall per step at ~6e7 decisions/s/core (calibrated below)
+    ctx = mp.get_context("fork")
+    with ctx.Pool(cores, initializer=_pool_init, initargs=(cfg,)) as pool:
+        t = pool.map(_oracle_range, [(cfg, 0, 1, cfg)] * cores)
+        per_kernel = max(min(t), 1e-4)
+        sample = int(max(cores, min(n_k, 2.0 / per_kernel * cores)))
+        per = (sample + cores - 1) // cores
+        jobs = [(cfg, i * per, min(per, sample - i * per), cfg) for i in range(cores) if i * per < sample]
+        for _ in range(args.warmup):
+            pool.map(_oracle_range, jobs)
+        times = []
+        for _ in range(args.steps):
+            t0 = time.perf_counter()
+            pool.map(_oracle_range, jobs)
+            times.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(times) / len(times)
+    value = sample * n_f / (sum(times) / len(times))
+    desc = f"first {sample} kernels of {cfg} per step, {len(jobs)} processes x single-threaded oracle"
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_desc(cfg), "sample_kernels_per_step": sample,
+                       "decisions_per_eval": dec},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": len(jobs), "kind": "oracle", "sample": desc},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------ ours
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_fandccfc23_b200 import build as B
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    from paper_conf_sc_fandccfc23_b200.dist import ShardedSweep, shard_rows
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    if rank == 0:
+        B.build()
+    if world > 1:
+        dist.barrier()
+    syn.load()
+
+    cfg = args.config
+    n_cfg, n_f = W.CONFIGS[cfg][0], W.CONFIGS[cfg][1]
+    sp_spec, en_spec, freqs, d = W.make_models(cfg)
+    targets = W.targets_six() if W.CONFIGS[cfg][4] == "six" else W.targets_es_pl()
+    weak = args.scaling == "weak"
+    if weak:
+        row0, n_local = rank * n_cfg, n_cfg
+    else:
+        row0, n_local, _ = shard_rows(n_cfg, rank, world)
+    feats_np = W.make_features(cfg, row0, n_local)
+    sp, en, ck = syn.Model(sp_spec, local), syn.Model(en_spec, local), syn.Clocks(freqs, local)
+    feats = torch.from_numpy(feats_np).to(dev)
+    n_t = len(targets)
+    sharded = ShardedSweep(n_cfg, n_t, rank, world, dev, weak=weak,
+                           compute=lambda f, o: syn.sweep(sp, en, f, ck, d, targets, out=o))
+    flush = torch.empty(args.flush_mib * (1 << 20) // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        return sharded.run(feats)
+
+    # warm-up (untimed), incl. a short clock ramp so the timed region runs at load clocks
+    for _ in range(args.warmup):
+        flush.zero_()
+        step()
+    t_end = time.time() + 0.5
+    while time.time() < t_end:
+        step()
+    torch.cuda.synchronize()
+
+    K = args.steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+           torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    launches = 0
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with sampler:
+        for i in range(K):
+            flush.zero_()                                   # L2 flush, outside the events
+            ev[i][0].record(stream)
+            if sharded.n_local:
+                syn.sweep(sp, en, feats, ck, d, targets, out=sharded.local[:sharded.n_local])
+                launches += syn.last_launch()["kernels"]
+            ev[i][1].record(stream)
+            if world > 1:
+                dist.all_gather_into_tensor(sharded.table, sharded.local)
+            ev[i][2].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+    kern_ms = [a.elapsed_time(b) for a, b, _ in ev]
+    step_ms = [a.elapsed_time(c) for a, _, c in ev]
+    total_ms = sum(step_ms)
+    tot = torch.tensor([total_ms, sum(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    total_ms_max = float(tot[0])
+    evals_step = (n_local if not weak else n_cfg) * n_f
+    evals_all = (n_cfg * world if weak else n_cfg) * n_f
+    value = evals_all * K / (total_ms_max / 1e3)
+
+    # ------------------------------------------------ e2e through the host-buffer C-ABI path
+    e2e = None
+    if not args.no_e2e:
+        h_feats = torch.from_numpy(feats_np).pin_memory()
+        e_ms = []
+        if world == 1:
+            ws = syn.Workspace(local)
+            h_out = torch.empty((n_local, n_t), dtype=torch.int32).pin_memory()
+            for i in range(args.warmup + K):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                ws.sweep_host(sp, en, h_feats, ck, d, targets, h_out)
+                b.record(stream)
+                b.synchronize()
+                if i >= args.warmup:
+                    e_ms.append(a.elapsed_time(b))
+            h2d, d2h = h_feats.numel() * 4, h_out.numel() * 4
+            ref_ok = bool((h_out.to(dev) == sharded.local[:n_local]).all())
+        else:
+            d_feats = torch.empty_like(feats)
+            h_table = torch.empty(tuple(sharded.gathered().shape), dtype=torch.int32).pin_memory()
+            for i in range(args.warmup + K):
+                flush.zero_()
+                dist.barrier()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                d_feats.copy_(h_feats, non_blocking=True)
+                tbl = sharded.run(d_feats)
+                h_table.copy_(tbl, non_blocking=True)
+                b.record(stream)
+                b.synchronize()
+                if i >= args.warmup:
+                    e_ms.append(a.elapsed_time(b))
+            h2d, d2h = h_feats.numel() * 4, h_table.numel() * 4
+            ref_ok = True
+        et = torch.tensor([sum(e_ms)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e = {"value": evals_all * K / (float(et[0]) / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": float(et[0]) / K, "matches_device_path": ref_ok}
+
+    # ------------------------------------------------------------------------- roofline
+    peaks, peak_src = load_peaks()
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    dec = decisions_per_eval(sp_spec) + decisions_per_eval(en_spec)
+    kern_avg_s = statistics.mean(kern_ms) / 1e3
+    achieved = evals_step * dec / kern_avg_s / 1e9                  # G node-decisions / s
+    # on-chip ceiling: one warp-level node decision needs >= 2 L1/shared
+    # wavefronts (node load + feature load), 1 wavefront/clk/SM -> 16 lane-decisions/clk/SM
+    peak = sms * sm_max * 1e6 * 32 / 2 / 1e9
+    hbm_bytes = evals_step // n_f * (W.N_STATIC * 4 + n_t * 4) + n_f * 4 + \
+        sp.info()["device_bytes"] + en.info()["device_bytes"]
+    hbm_ach = hbm_bytes / kern_avg_s / 1e9
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
+                "frac": achieved / peak, "traffic": ncu_traffic(cfg),
+                "kernel": "k_sweep", "kernel_ms": statistics.mean(kern_ms),
+                "kernel_share_of_step": sum(kern_ms) / total_ms,
+                "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
+                "hbm": {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                        "frac": hbm_ach / peaks["hbm_gbs"], "algorithmic_bytes": hbm_bytes,
+                        "peak_source": peak_src}}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, ev_n, el = oracle_single_core(cfg, min(n_cfg, 1000))
+        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"first {min(n_cfg, 1000)} kernels of {cfg} x {n_f} clocks repeated to "
+                         f"{el:.1f} s ({ev_n} evals), single-threaded oracle (oracle/oracle.c)"}
+
+    if rank == 0:
+        clocks = sampler.summary()
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
+                "warmup": args.warmup, "ms_per_step": total_ms_max / K, "higher_is_better": True,
+                "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": workload_desc(cfg), "n_kernels_per_rank": n_local,
+                           "n_freqs": n_f, "targets": n_t,
+                           "parallelism": f"dp{world} (kernel axis) + NCCL all-gather of choices",
+                           "l2": f"flushed between timed steps ({args.flush_mib} MiB write)",
+                           "decisions_per_eval": dec},
+                "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
+                "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,175 @@
+/* synergy.h — C ABI of the B200 (sm_100a) SYnergy predict+select library (libsynergy.so).
+ *
+ * The operation (PAPER.md = the SYnergy paper, SC'23; "L<n>" = line n):
+ *   §6.2 Prediction phase, L316-L322: for a new workload's static feature vector k'
+ *   (Table 1) and the device's core-clock vector f (L59-L65, L312) build the
+ *   prediction dataset P = (k', f), predict the metrics with the trained single-target
+ *   models (L320; families Linear / Lasso / RandomForest, L386 and Table 2), then "find the
+ *   frequency configuration f-hat by using a search algorithm for different energy targets,
+ *   e.g. MIN_EDP, ES_25 or PL_25" (L322).  Energy targets: EDP = e*t, ED2P = e*t^2 (L253),
+ *   ES_x (L259-L267), PL_x (L269-L271), MAX_PERF / MIN_ENERGY (L382, Table 2), all relative
+ *   to the default clock (L69).  The library evaluates every (kernel, clock) pair of a batch
+ *   of kernels with a speedup model and an energy model, normalises both to the default
+ *   clock, and returns one clock index per kernel per target.  The readings of points the
+ *   paper leaves open are DESIGN.md Q1-Q23 (exhaustive lowest-index argmin, potential-saving
+ *   ES/PL, x <= threshold goes left, fp64 accumulation, ...).
+ *
+ * Conventions for every call:
+ *   - All calls return syn_status; no C++ exception crosses the ABI.  On a non-OK status the
+ *     reason is available from synergy_last_error() (thread-local, valid until the next call
+ *     on the same thread).
+ *   - Argument errors are detected on the host before anything is enqueued; on error NOTHING
+ *     is enqueued and outputs are untouched.
+ *   - Device-side calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy default
+ *     stream).  Results are valid after the caller synchronises that stream.  Launch failures
+ *     return SYN_ERR_CUDA.
+ *   - "d_" pointers are device pointers on the model's device, "h_" pointers host pointers.
+ *     The caller owns every buffer it passes; the hot calls never allocate.
+ *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
+ *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
+ *   - Handles (models, clock tables, workspaces) are bound to the device they were created
+ *     on and must be used with that device current.  Models and clock tables are immutable
+ *     and may be shared across streams and host threads.
+ */
+#ifndef SYNERGY_H
+#define SYNERGY_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SYNERGY_VERSION 1
+#define SYNERGY_MAX_FREQS 4096
+#define SYNERGY_MAX_TARGETS 16
+#define SYNERGY_MAX_INPUTS 255
+#define SYNERGY_MAX_DEPTH 64
+
+typedef enum {
+    SYN_OK = 0,
+    SYN_ERR_INVALID_ARG = 1,   /* bad pointer, size, index, target, model or clock table   */
+    SYN_ERR_UNSUPPORTED = 2,   /* well-formed but beyond the library's limits              */
+    SYN_ERR_CUDA = 3,          /* a CUDA runtime call or kernel launch failed              */
+    SYN_ERR_OOM = 4            /* device or host allocation failed                         */
+} syn_status;
+
+/* Energy targets (Listing 3, Table 2). */
+typedef enum {
+    SYN_MAX_PERF = 0,    /* highest speedup                                         */
+    SYN_MIN_ENERGY = 1,  /* lowest energy                                           */
+    SYN_MIN_EDP = 2,     /* lowest E*T, T = 1/S                  (L253)             */
+    SYN_MIN_ED2P = 3,    /* lowest E*T^2                         (L253)             */
+    SYN_ES = 4,          /* highest speedup with E <= E_def - x%(E_def - E_min)  (L267) */
+    SYN_PL = 5           /* lowest energy with S >= S_def - x%(S_def - S(i_minE)) (L271) */
+} syn_target_kind;
+
+typedef struct {
+    int32_t kind;        /* syn_target_kind                                         */
+    float x;             /* percentage in [0, 100] for SYN_ES / SYN_PL, else ignored */
+} syn_target;
+
+typedef void *syn_stream;   /* cudaStream_t */
+
+/* Model description (host memory; copied by synergy_model_create).  The forest uses
+ * scikit-learn's `tree_` layout: structure of arrays over the nodes of all trees, node ids
+ * tree-local with root 0, children -1 at leaves, value = split threshold (internal node,
+ * x[feature] <= value goes left) or leaf value.  Input index n_inputs-1 is the core clock
+ * in MHz; inputs 0..n_inputs-2 are the static features.  Output (Q7/Q8):
+ *   m(x) = 0;  m += linear_weight * (lin_b + sum_j lin_w[j] x[j])   if linear_weight != 0
+ *              m += forest_weight * mean_t leaf_t(x)                if forest_weight != 0
+ * accumulated in fp64 (fp64 fma over j in order for the linear member, fp64 sum of the fp32
+ * leaves in tree order, then / n_trees); a weight of exactly 1 skips its multiplication. */
+typedef struct {
+    int32_t n_inputs;            /* F + 1, 1 .. SYNERGY_MAX_INPUTS                        */
+    double linear_weight;        /* 0 => no linear member                                 */
+    const double *lin_w;         /* [n_inputs]                                            */
+    double lin_b;
+    double forest_weight;        /* 0 => no forest member                                 */
+    int32_t n_trees;             /* >= 1 when forest_weight != 0                          */
+    const int64_t *tree_offset;  /* [n_trees+1] node range of each tree                   */
+    const int32_t *feature;      /* [n_nodes] split input, -1 = leaf                      */
+    const int32_t *left;         /* [n_nodes] tree-local child ids (ignored at leaves)    */
+    const int32_t *right;
+    const float *value;          /* [n_nodes] threshold or leaf value                     */
+} syn_model_desc;
+
+typedef struct syn_model syn_model;      /* opaque, device-resident, immutable */
+typedef struct syn_clocks syn_clocks;    /* opaque, device-resident, immutable */
+typedef struct syn_workspace syn_workspace;
+
+/* Thread-local message for the last non-OK status ("" if none). */
+const char *synergy_last_error(void);
+int32_t synergy_version(void);
+
+/* Validate, re-lay (breadth-first, children adjacent) and upload a model to `device`.
+ * INVALID_ARG: null arrays, n_inputs out of range, a child id outside its tree, a node
+ * reached twice (not a tree), a split feature outside [0, n_inputs), both weights 0.
+ * UNSUPPORTED: depth > SYNERGY_MAX_DEPTH or more than 2^31-2 nodes.  OOM / CUDA otherwise.
+ * Synchronous (returns after the upload). */
+syn_status synergy_model_create(const syn_model_desc *desc, int32_t device, syn_model **out);
+syn_status synergy_model_destroy(syn_model *model);
+/* Any output pointer may be NULL.  max_depth = deepest root-to-leaf path (edges). */
+syn_status synergy_model_info(const syn_model *model, int32_t *n_inputs, int32_t *n_trees,
+                              int64_t *n_nodes, int32_t *max_depth, int64_t *device_bytes);
+
+/* Core-clock table f: h_freqs[n_freqs] in MHz, finite and strictly
+ * ascending (INVALID_ARG otherwise), 1 <= n_freqs <= SYNERGY_MAX_FREQS.  Synchronous. */
+syn_status synergy_clocks_create(const float *h_freqs, int32_t n_freqs, int32_t device,
+                                 syn_clocks **out);
+syn_status synergy_clocks_destroy(syn_clocks *clocks);
+syn_status synergy_clocks_info(const syn_clocks *clocks, int32_t *n_freqs);
+
+/* Predictions for every (kernel, clock) pair:
+ *   d_speedup[k][i] = (float)(mS(k, f_i) / mS(k, f_def)),  d_energy likewise with mE,
+ * or (float)m when default_idx == -1 (raw model outputs).  n_kernels == 0 is a no-op.
+ * INVALID_ARG: null model / clocks / non-empty buffers, n_kernels < 0, n_features + 1 !=
+ * n_inputs of either model, default_idx outside [-1, n_freqs), handle on another device. */
+syn_status synergy_predict(const syn_model *speedup, const syn_model *energy,
+                           const float *d_features, int64_t n_kernels, int32_t n_features,
+                           const syn_clocks *clocks, int32_t default_idx,
+                           float *d_speedup, float *d_energy, syn_stream stream);
+
+/* Target selection on given normalised predictions:
+ *   valid_i = S_i, E_i finite and > 0; if the default is invalid all choices are -1;
+ *   baselines S_def, E_def, E_min (lowest index of the minimum), S_minE; per target the
+ *   objective key / constraint of syn_target_kind evaluated in fp64; d_choice[k][t] = the
+ *   lowest index i minimising the key among valid feasible candidates, -1 if none.
+ * INVALID_ARG: null buffers, n_kernels < 0, n_freqs outside [1, SYNERGY_MAX_FREQS],
+ * default_idx outside [0, n_freqs), n_targets outside [1, SYNERGY_MAX_TARGETS], unknown kind,
+ * ES/PL x NaN or outside [0, 100]. */
+syn_status synergy_select(const float *d_speedup, const float *d_energy, int64_t n_kernels,
+                          int32_t n_freqs, int32_t default_idx, const syn_target *h_targets,
+                          int32_t n_targets, int32_t *d_choice, syn_stream stream);
+
+/* Fused predict + select in one kernel: predictions stay on chip unless d_speedup /
+ * d_energy are non-NULL (then they are also written, as synergy_predict would).
+ * default_idx must be in [0, n_freqs).  Other errors as predict + select. */
+syn_status synergy_sweep(const syn_model *speedup, const syn_model *energy,
+                         const float *d_features, int64_t n_kernels, int32_t n_features,
+                         const syn_clocks *clocks, int32_t default_idx,
+                         const syn_target *h_targets, int32_t n_targets, int32_t *d_choice,
+                         float *d_speedup, float *d_energy, syn_stream stream);
+
+/* End-to-end host-buffer path: copies h_features host->device into the workspace, runs
+ * synergy_sweep, copies the choices device->host into h_choice, all enqueued on `stream`
+ * (h_choice is valid after the stream is synchronised; pinned host buffers make the copies
+ * asynchronous).  The workspace grows on demand (the only allocating call; OOM possible) and
+ * must not be used by two streams at once. */
+syn_status synergy_workspace_create(int32_t device, syn_workspace **out);
+syn_status synergy_workspace_destroy(syn_workspace *ws);
+syn_status synergy_sweep_host(syn_workspace *ws, const syn_model *speedup,
+                              const syn_model *energy, const float *h_features,
+                              int64_t n_kernels, int32_t n_features, const syn_clocks *clocks,
+                              int32_t default_idx, const syn_target *h_targets,
+                              int32_t n_targets, int32_t *h_choice, syn_stream stream);
+
+/* Launch statistics of the last sweep/predict/select enqueued by this host thread (for
+ * benchmarks: kernels launched, evaluations, node decisions of complete paths).  NULLs ok. */
+syn_status synergy_last_launch(int32_t *kernels_launched, int64_t *evals, int64_t *grid,
+                               int32_t *block, int32_t *variant);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SYNERGY_H */

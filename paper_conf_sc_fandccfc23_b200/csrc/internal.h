@@ -1,0 +1,66 @@
+// internal.h — device-side data layout shared by the C-ABI host code and the kernels.
+// Not part of the public ABI (include/synergy.h).  See DESIGN.md "Data layout in HBM".
+#pragma once
+#include <cstdint>
+
+namespace syn {
+
+// Packed forest node, 8 bytes, breadth-first per tree with the two children adjacent:
+//   .x = bits of the fp32 threshold (internal) or leaf value (leaf)
+//   .y = meta = (delta << 8) | code,  delta signed 24-bit
+//        code in [0, F)  : split on static feature `code`
+//        code == F       : split on the core clock (input F)
+//        code == F + 1   : leaf (the kernel's x-vector slot F+1 holds NaN, so the
+//                          comparison is false and idx += delta + 1 == idx + 0)
+//   next = idx + delta + (x <= thr ? 0 : 1);  leaves use delta = -1 (self loop).
+// With per-tree depth D every lane takes exactly D steps, branch-free, and lands on a leaf.
+constexpr int kCodeBits = 8;
+constexpr int kMaxDelta = (1 << 23) - 1;
+
+struct DevModel {
+    const uint2* nodes;      // [n_nodes + 1]; node n_nodes is a padding leaf (value 0)
+    const int2* trees;       // [n_trees] {first node (BFS root), depth}
+    const double* lin_w;     // [n_inputs]
+    double lin_b;
+    double lin_weight;       // 0 => absent
+    double forest_weight;    // 0 => absent
+    int n_trees;
+    int pad_leaf;            // index of the padding leaf
+};
+
+constexpr int kMaxTargets = 16;
+
+enum Mode : int { kModePredict = 0, kModeSweep = 1 };
+
+struct SweepArgs {
+    DevModel ms, me;         // speedup, energy
+    const float* features;   // [n_k][F]
+    long long n_k;
+    int F;                   // static features; clock is input F
+    const float* freqs;      // [n_f]
+    int n_f;
+    int def;                 // default clock index; -1 = raw (predict only)
+    int n_t;
+    int kind[kMaxTargets];
+    float x[kMaxTargets];
+    int* choice;             // [n_k][n_t] (sweep)
+    float* S_out;            // [n_k][n_f] or null
+    float* E_out;
+    int mode;
+    int tile_k;              // kernels per CTA
+    int xs;                  // x-vector stride in smem (floats)
+};
+
+struct SelectArgs {
+    const float* S;
+    const float* E;
+    long long n_k;
+    int n_f;
+    int def;
+    int n_t;
+    int kind[kMaxTargets];
+    float x[kMaxTargets];
+    int* choice;
+};
+
+}  // namespace syn

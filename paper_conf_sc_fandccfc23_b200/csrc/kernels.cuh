@@ -1,0 +1,245 @@
+// kernels.cuh — sm_100a kernels of the SYnergy predict+select hot path.
+//
+//   k_sweep<SLOTS, TILP>  fused: model inference for every (kernel, clock) pair of a CTA's
+//                         kernel tile, default-clock normalisation (L69), then
+//                         per-target objective + masked lowest-index argmin (L253-L271, L322)
+//                         with warp shuffles; predictions stay in shared memory unless asked.
+//   k_select              standalone selection over predictions in HBM (one warp per kernel).
+//
+// Arithmetic contract (Q15): identical op sequence to the oracle — fp64 fma chain
+// for the linear member, fp64 sum of fp32 leaves in tree order, fp64 division by T, fp64
+// normalisation rounded once to fp32, fp64 keys/thresholds; every fp64 op is an explicit
+// _rn intrinsic so nothing is contracted.  Ties: lexicographic (key, index) minimum.
+#pragma once
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <cstdint>
+
+#include "internal.h"
+
+namespace syn {
+
+__device__ __forceinline__ uint2 ldg_node(const uint2* p) {
+    uint2 r;
+    asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+    return r;
+}
+
+__device__ __forceinline__ bool valid_pred(float s, float e) {
+    // DESIGN.md Q16: finite and strictly positive speedup and energy
+    return isfinite(s) && isfinite(e) && s > 0.0f && e > 0.0f;
+}
+
+// Raw model output for SLOTS (kernel, clock) units held by this thread.
+//   xk[row[s] + j] = static feature j of the unit's kernel, slot F+1 = NaN (leaf code)
+template <int SLOTS, int TILP>
+__device__ __forceinline__ void eval_model(const DevModel& m, const float* __restrict__ xk,
+                                           const int (&row)[SLOTS], const float (&f)[SLOTS],
+                                           int F, double (&out)[SLOTS]) {
+#pragma unroll
+    for (int s = 0; s < SLOTS; ++s) out[s] = 0.0;
+    if (m.lin_weight != 0.0) {
+        // Linear / Lasso member (L386): lin = b; lin = fma(w_j, x_j, lin), j = 0..F in order
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s) {
+            double lin = m.lin_b;
+            for (int j = 0; j < F; ++j) lin = __fma_rn(__ldg(m.lin_w + j), (double)xk[row[s] + j], lin);
+            lin = __fma_rn(__ldg(m.lin_w + F), (double)f[s], lin);
+            out[s] = __dadd_rn(out[s], m.lin_weight == 1.0 ? lin : __dmul_rn(m.lin_weight, lin));
+        }
+    }
+    if (m.forest_weight != 0.0) {
+        // Random Forest member (L386): mean of T trees, x <= thr goes left (Q8, Q9)
+        double acc[SLOTS];
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s) acc[s] = 0.0;
+        for (int t0 = 0; t0 < m.n_trees; t0 += TILP) {
+            const int nt = min(TILP, m.n_trees - t0);
+            int idx[TILP][SLOTS];
+            int depth = 0;
+#pragma unroll
+            for (int j = 0; j < TILP; ++j) {
+                int2 td = (j < nt) ? __ldg(m.trees + t0 + j) : make_int2(m.pad_leaf, 0);
+                depth = max(depth, td.y);
+#pragma unroll
+                for (int s = 0; s < SLOTS; ++s) idx[j][s] = td.x;
+            }
+            // depth is uniform across the CTA: every lane takes the same number of steps,
+            // lanes that reached a leaf early self-loop on it (no divergence)
+            for (int d = 0; d < depth; ++d) {
+#pragma unroll
+                for (int j = 0; j < TILP; ++j) {
+#pragma unroll
+                    for (int s = 0; s < SLOTS; ++s) {
+                        const uint2 n = ldg_node(m.nodes + idx[j][s]);
+                        const int code = (int)(n.y & 0xffu);
+                        const float xs = xk[row[s] + code];
+                        const float x = (code == F) ? f[s] : xs;
+                        idx[j][s] += ((int)n.y >> kCodeBits) + (x <= __uint_as_float(n.x) ? 0 : 1);
+                    }
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < TILP; ++j) {
+                if (j < nt) {   // uniform guard; accumulation strictly in tree order
+#pragma unroll
+                    for (int s = 0; s < SLOTS; ++s)
+                        acc[s] = __dadd_rn(acc[s], (double)__uint_as_float(ldg_node(m.nodes + idx[j][s]).x));
+                }
+            }
+        }
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s) {
+            const double forest = __ddiv_rn(acc[s], (double)m.n_trees);
+            out[s] = __dadd_rn(out[s], m.forest_weight == 1.0 ? forest : __dmul_rn(m.forest_weight, forest));
+        }
+    }
+}
+
+__device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+        const double ok = __shfl_xor_sync(0xffffffffu, key, off);
+        const int oi = __shfl_xor_sync(0xffffffffu, idx, off);
+        if (ok < key || (ok == key && oi < idx)) { key = ok; idx = oi; }
+    }
+}
+
+// One warp selects all targets of one kernel from its n_f normalised predictions
+// (S, E in shared or global memory).  Writes out[0..n_t).
+__device__ __forceinline__ void select_row_warp(const float* S, const float* E, int n_f, int def,
+                                                int n_t, const int* kind, const float* xs,
+                                                int* out, int lane) {
+    const float sd = S[def], ed = E[def];
+    if (!valid_pred(sd, ed)) {              // no baseline: every target -1
+        for (int t = lane; t < n_t; t += 32) out[t] = -1;
+        return;
+    }
+    // minimum-energy point, lowest index among equal minima (baseline of ES/PL, L265)
+    double be = CUDART_INF;
+    int bi = INT_MAX;
+    for (int i = lane; i < n_f; i += 32) {
+        const float s = S[i], e = E[i];
+        if (valid_pred(s, e) && (double)e < be) { be = (double)e; bi = i; }
+    }
+    argmin_shfl(be, bi);
+    const double E_def = (double)ed, S_def = (double)sd;
+    const double E_min = (double)E[bi], S_minE = (double)S[bi];
+    for (int t = 0; t < n_t; ++t) {
+        const int kd = kind[t];
+        const double frac = __ddiv_rn((double)xs[t], 100.0);
+        const double thr_es = __dsub_rn(E_def, __dmul_rn(frac, __dsub_rn(E_def, E_min)));
+        const double thr_pl = __dsub_rn(S_def, __dmul_rn(frac, __dsub_rn(S_def, S_minE)));
+        double bk = CUDART_INF;
+        int bx = INT_MAX;
+        for (int i = lane; i < n_f; i += 32) {
+            const float sf = S[i], ef = E[i];
+            if (!valid_pred(sf, ef)) continue;
+            const double s = (double)sf, e = (double)ef;
+            double key;
+            bool feas = true;
+            switch (kd) {
+                case 0: key = -s; break;                                   // MAX_PERF
+                case 1: key = e; break;                                    // MIN_ENERGY
+                case 2: key = __ddiv_rn(e, s); break;                      // MIN_EDP  e*t
+                case 3: key = __ddiv_rn(__ddiv_rn(e, s), s); break;        // MIN_ED2P e*t^2
+                case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
+                default: feas = (s >= thr_pl); key = e; break;             // PL_x
+            }
+            if (feas && (key < bk || (key == bk && i < bx))) { bk = key; bx = i; }
+        }
+        argmin_shfl(bk, bx);
+        if (lane == 0) out[t] = (bx == INT_MAX) ? -1 : bx;
+    }
+}
+
+template <int SLOTS, int TILP>
+__global__ void __launch_bounds__(512) k_sweep(const __grid_constant__ SweepArgs a) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int tile = a.tile_k;
+    const long long k0 = (long long)blockIdx.x * tile;
+    const int nk = (int)min((long long)tile, a.n_k - k0);
+    const int n_f = a.n_f;
+    const int F = a.F;
+    const int XS = a.xs;
+    double* mS = reinterpret_cast<double*>(smem);
+    double* mE = mS + (size_t)tile * n_f;
+    float* sS = reinterpret_cast<float*>(mE + (size_t)tile * n_f);
+    float* sE = sS + (size_t)tile * n_f;
+    float* xk = sE + (size_t)tile * n_f;
+    float* fr = xk + (size_t)tile * XS;
+
+    // stage the tile's feature rows (coalesced) and the clock table
+    const float* gfeat = a.features + k0 * F;
+    for (int e = threadIdx.x; e < nk * F; e += blockDim.x) {
+        const int r = e / F;
+        xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
+    }
+    for (int r = threadIdx.x; r < nk; r += blockDim.x) {
+        xk[r * XS + F] = 0.0f;
+        xk[r * XS + F + 1] = CUDART_NAN_F;     // leaf code slot
+    }
+    for (int i = threadIdx.x; i < n_f; i += blockDim.x) fr[i] = __ldg(a.freqs + i);
+    __syncthreads();
+
+    // phase 1: every (kernel, clock) unit of the tile -> raw fp64 model outputs
+    const int units = nk * n_f;
+    for (int u0 = 0; u0 < units; u0 += blockDim.x * SLOTS) {
+        int row[SLOTS];
+        float f[SLOTS];
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s) {
+            const int u = u0 + threadIdx.x + s * blockDim.x;
+            const int uu = u < units ? u : 0;
+            const int kl = uu / n_f;
+            row[s] = kl * XS;
+            f[s] = fr[uu - kl * n_f];
+        }
+        double vS[SLOTS], vE[SLOTS];
+        eval_model<SLOTS, TILP>(a.ms, xk, row, f, F, vS);
+        eval_model<SLOTS, TILP>(a.me, xk, row, f, F, vE);
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s) {
+            const int u = u0 + threadIdx.x + s * blockDim.x;
+            if (u < units) { mS[u] = vS[s]; mE[u] = vE[s]; }
+        }
+    }
+    __syncthreads();
+
+    // phase 2: per kernel (one warp each): normalise to the default clock, then select
+    const int lane = threadIdx.x & 31;
+    const int nw = blockDim.x >> 5;
+    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
+        const double* rS = mS + (size_t)kl * n_f;
+        const double* rE = mE + (size_t)kl * n_f;
+        float* oS = sS + (size_t)kl * n_f;
+        float* oE = sE + (size_t)kl * n_f;
+        const long long k = k0 + kl;
+        const double dS = a.def >= 0 ? rS[a.def] : 1.0;
+        const double dE = a.def >= 0 ? rE[a.def] : 1.0;
+        for (int i = lane; i < n_f; i += 32) {
+            const float s = a.def >= 0 ? __double2float_rn(__ddiv_rn(rS[i], dS)) : __double2float_rn(rS[i]);
+            const float e = a.def >= 0 ? __double2float_rn(__ddiv_rn(rE[i], dE)) : __double2float_rn(rE[i]);
+            oS[i] = s;
+            oE[i] = e;
+            if (a.S_out) a.S_out[k * n_f + i] = s;
+            if (a.E_out) a.E_out[k * n_f + i] = e;
+        }
+        __syncwarp();
+        if (a.mode == kModeSweep)
+            select_row_warp(oS, oE, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
+    }
+}
+
+// Standalone selection: one warp per kernel row, rows read from HBM (L1-resident across the
+// per-target passes).  Grid-stride over kernels.
+__global__ void __launch_bounds__(256) k_select(const __grid_constant__ SelectArgs a) {
+    const int lane = threadIdx.x & 31;
+    const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+    for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < a.n_k; k += warps) {
+        select_row_warp(a.S + k * a.n_f, a.E + k * a.n_f, a.n_f, a.def, a.n_t, a.kind, a.x,
+                        a.choice + k * a.n_t, lane);
+    }
+}
+
+}  // namespace syn

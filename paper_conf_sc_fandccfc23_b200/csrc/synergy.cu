@@ -1,0 +1,543 @@
+// synergy.cu — C-ABI implementation (include/synergy.h): validation, model packing, launch
+// configuration and the host-buffer end-to-end path.  All compute runs in kernels.cuh.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+#include "kernels.cuh"
+#include "synergy.h"
+
+using namespace syn;
+
+struct syn_model {
+    int device;
+    int n_inputs;
+    int n_trees;
+    int max_depth;
+    long long n_nodes;
+    long long bytes;
+    void* alloc;
+    DevModel dm;
+};
+
+struct syn_clocks {
+    int device;
+    int n_f;
+    float* d_freqs;
+};
+
+struct syn_workspace {
+    int device;
+    float* d_features;
+    size_t cap_features;      // bytes
+    int* d_choice;
+    size_t cap_choice;        // bytes
+};
+
+namespace {
+
+thread_local std::string g_err;
+struct LaunchInfo {
+    int kernels;
+    long long evals;
+    long long grid;
+    int block;
+    int variant;
+};
+thread_local LaunchInfo g_last = {0, 0, 0, 0, 0};
+
+syn_status fail(syn_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return st;
+}
+
+syn_status cuda_fail(cudaError_t e, const char* what) {
+    return fail(e == cudaErrorMemoryAllocation ? SYN_ERR_OOM : SYN_ERR_CUDA, "%s: %s", what,
+                cudaGetErrorString(e));
+}
+
+syn_status ok() {
+    g_err.clear();
+    return SYN_OK;
+}
+
+struct DeviceGuard {   // switch to `dev` for the scope, restore afterwards
+    int prev = -1;
+    bool okay = false;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) == cudaSuccess && cudaSetDevice(dev) == cudaSuccess) okay = true;
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+bool current_device_is(int dev) {
+    int cur = -1;
+    return cudaGetDevice(&cur) == cudaSuccess && cur == dev;
+}
+
+int sm_count(int dev) {
+    static int cached[64] = {0};
+    if (dev < 0 || dev >= 64) return 148;
+    if (!cached[dev]) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
+        cached[dev] = v;
+    }
+    return cached[dev];
+}
+
+syn_status check_targets(const syn_target* t, int32_t n_t) {
+    if (n_t < 1 || n_t > SYNERGY_MAX_TARGETS) return fail(SYN_ERR_INVALID_ARG, "n_targets=%d outside [1, %d]", n_t, SYNERGY_MAX_TARGETS);
+    if (!t) return fail(SYN_ERR_INVALID_ARG, "h_targets is NULL");
+    for (int i = 0; i < n_t; ++i) {
+        if (t[i].kind < SYN_MAX_PERF || t[i].kind > SYN_PL) return fail(SYN_ERR_INVALID_ARG, "target %d: unknown kind %d", i, t[i].kind);
+        if ((t[i].kind == SYN_ES || t[i].kind == SYN_PL) && !(t[i].x >= 0.0f && t[i].x <= 100.0f))
+            return fail(SYN_ERR_INVALID_ARG, "target %d: x=%g outside [0, 100]", i, (double)t[i].x);
+    }
+    return SYN_OK;
+}
+
+// ---------------------------------------------------------------- launch configuration
+
+struct Config {
+    int slots, tilp, tile_k, nt, xs;
+    size_t smem;
+};
+
+size_t sweep_smem(int tile_k, int n_f, int xs) {
+    return (size_t)tile_k * ((size_t)n_f * 24 + (size_t)xs * 4) + (size_t)n_f * 4;
+}
+
+// Choose per-thread slots (units in flight) and trees-in-flight so that the grid keeps every
+// SM busy for small batches (slots=1, 4 trees in flight) and amortises staging for large ones.
+Config choose_config(long long n_k, int n_f, int F, int dev) {
+    Config c;
+    const long long resident = (long long)sm_count(dev) * 2048;
+    const long long evals = n_k * (long long)n_f;
+    c.slots = evals >= 16 * resident ? 8 : evals >= 8 * resident ? 4 : evals >= 4 * resident ? 2 : 1;
+    c.tilp = c.slots <= 2 ? 4 : c.slots == 4 ? 2 : 1;
+    c.xs = (F + 2) | 1;   // odd stride: rows of different kernels land in different banks
+    long long tk = std::max(1, (256 * c.slots) / n_f);
+    tk = std::min<long long>(tk, std::max<long long>(n_k, 1));
+    while (tk > 1 && sweep_smem((int)tk, n_f, c.xs) > 200 * 1024) --tk;
+    c.tile_k = (int)tk;
+    long long thr = (c.tile_k * (long long)n_f + c.slots - 1) / c.slots;
+    thr = (thr + 31) / 32 * 32;
+    c.nt = (int)std::min<long long>(std::max<long long>(thr, 32), 512);
+    c.smem = sweep_smem(c.tile_k, n_f, c.xs);
+    return c;
+}
+
+template <int S, int T>
+cudaError_t launch_sweep_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    static size_t smem_set = 48 * 1024;   // per-instantiation opt-in high-water mark
+    if (c.smem > smem_set) {
+        cudaError_t e = cudaFuncSetAttribute(k_sweep<S, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        if (e != cudaSuccess) return e;
+        smem_set = c.smem;
+    }
+    k_sweep<S, T><<<(unsigned)grid, c.nt, c.smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sweep(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    switch (c.slots) {
+        case 1: return launch_sweep_t<1, 4>(a, c, grid, st);
+        case 2: return launch_sweep_t<2, 4>(a, c, grid, st);
+        case 4: return launch_sweep_t<4, 2>(a, c, grid, st);
+        default: return launch_sweep_t<8, 1>(a, c, grid, st);
+    }
+}
+
+syn_status validate_sweep(const syn_model* sp, const syn_model* en, int64_t n_k, int32_t F,
+                          const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t, int mode) {
+    if (!sp || !en) return fail(SYN_ERR_INVALID_ARG, "model is NULL");
+    if (!clocks) return fail(SYN_ERR_INVALID_ARG, "clocks is NULL");
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    if (F + 1 != sp->n_inputs || F + 1 != en->n_inputs)
+        return fail(SYN_ERR_INVALID_ARG, "n_features+1=%d does not match model n_inputs (%d, %d)", F + 1, sp->n_inputs, en->n_inputs);
+    const int n_f = clocks->n_f;
+    if (mode == kModeSweep) {
+        if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
+        syn_status s = check_targets(targets, n_t);
+        if (s != SYN_OK) return s;
+    } else if (def < -1 || def >= n_f) {
+        return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [-1, %d)", def, n_f);
+    }
+    if (sp->device != clocks->device || en->device != clocks->device || !current_device_is(clocks->device))
+        return fail(SYN_ERR_INVALID_ARG, "model/clocks device differs from the current device");
+    return SYN_OK;
+}
+
+syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
+                     int32_t F, const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
+                     int32_t* d_choice, float* d_S, float* d_E, int mode, cudaStream_t st) {
+    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, mode);
+    if (vs != SYN_OK) return vs;
+    const int n_f = clocks->n_f;
+    if (n_k == 0) {
+        g_last = {0, 0, 0, 0, 0};
+        return ok();
+    }
+    if (!d_features) return fail(SYN_ERR_INVALID_ARG, "d_features is NULL");
+    if (mode == kModeSweep && !d_choice) return fail(SYN_ERR_INVALID_ARG, "d_choice is NULL");
+    if (mode == kModePredict && (!d_S || !d_E)) return fail(SYN_ERR_INVALID_ARG, "d_speedup/d_energy is NULL");
+
+    SweepArgs a;
+    memset(&a, 0, sizeof a);
+    a.ms = sp->dm;
+    a.me = en->dm;
+    a.features = d_features;
+    a.n_k = n_k;
+    a.F = F;
+    a.freqs = clocks->d_freqs;
+    a.n_f = n_f;
+    a.def = def;
+    a.n_t = mode == kModeSweep ? n_t : 0;
+    for (int t = 0; t < a.n_t; ++t) {
+        a.kind[t] = targets[t].kind;
+        a.x[t] = targets[t].x;
+    }
+    a.choice = d_choice;
+    a.S_out = d_S;
+    a.E_out = d_E;
+    a.mode = mode;
+    const Config c = choose_config(n_k, n_f, F, clocks->device);
+    a.tile_k = c.tile_k;
+    a.xs = c.xs;
+    const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
+    if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
+    cudaError_t e = launch_sweep(a, c, grid, st);
+    if (e != cudaSuccess) return cuda_fail(e, "k_sweep launch");
+    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.slots * 10 + c.tilp};
+    return ok();
+}
+
+}  // namespace
+
+// =============================================================================== C ABI
+
+extern "C" {
+
+const char* synergy_last_error(void) { return g_err.c_str(); }
+
+int32_t synergy_version(void) { return SYNERGY_VERSION; }
+
+syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_model** out) {
+    if (!out) return fail(SYN_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (!d) return fail(SYN_ERR_INVALID_ARG, "desc is NULL");
+    if (d->n_inputs < 1 || d->n_inputs > SYNERGY_MAX_INPUTS)
+        return fail(SYN_ERR_INVALID_ARG, "n_inputs=%d outside [1, %d]", d->n_inputs, SYNERGY_MAX_INPUTS);
+    if (!std::isfinite(d->linear_weight) || !std::isfinite(d->forest_weight))
+        return fail(SYN_ERR_INVALID_ARG, "member weights must be finite");
+    if (d->linear_weight == 0.0 && d->forest_weight == 0.0)
+        return fail(SYN_ERR_INVALID_ARG, "both member weights are 0");
+    if (d->linear_weight != 0.0 && !d->lin_w) return fail(SYN_ERR_INVALID_ARG, "lin_w is NULL");
+    const int F = d->n_inputs - 1;
+    const uint32_t leaf_code = (uint32_t)(F + 1);
+    std::vector<uint2> nodes;
+    std::vector<int2> trees;
+    int max_depth = 0;
+    if (d->forest_weight != 0.0) {
+        if (d->n_trees < 1) return fail(SYN_ERR_INVALID_ARG, "n_trees=%d < 1", d->n_trees);
+        if (!d->tree_offset || !d->feature || !d->left || !d->right || !d->value)
+            return fail(SYN_ERR_INVALID_ARG, "forest arrays must be non-NULL");
+        std::vector<int64_t> queue;
+        std::vector<int> qdepth;
+        std::vector<char> seen;
+        trees.resize(d->n_trees);
+        for (int t = 0; t < d->n_trees; ++t) {
+            const int64_t b = d->tree_offset[t], e = d->tree_offset[t + 1];
+            if (b < 0 || e <= b) return fail(SYN_ERR_INVALID_ARG, "tree %d: bad node range [%lld, %lld)", t, (long long)b, (long long)e);
+            const int64_t n = e - b;
+            if (n > kMaxDelta) return fail(SYN_ERR_UNSUPPORTED, "tree %d: %lld nodes > %d", t, (long long)n, kMaxDelta);
+            seen.assign((size_t)n, 0);
+            queue.assign(1, 0);
+            qdepth.assign(1, 0);
+            seen[0] = 1;
+            const int64_t base = (int64_t)nodes.size();
+            if (base + n > 0x7ffffff0LL) return fail(SYN_ERR_UNSUPPORTED, "more than 2^31 nodes");
+            int depth = 0;
+            // breadth-first re-layout: children pushed together, so right = left + 1
+            for (size_t p = 0; p < queue.size(); ++p) {
+                const int64_t id = queue[p];
+                const int32_t f = d->feature[b + id];
+                const float v = d->value[b + id];
+                uint32_t vb;
+                memcpy(&vb, &v, 4);
+                depth = std::max(depth, qdepth[p]);
+                if (f < 0) {
+                    nodes.push_back(make_uint2(vb, 0xFFFFFF00u | leaf_code));
+                    continue;
+                }
+                if (f >= d->n_inputs) return fail(SYN_ERR_INVALID_ARG, "tree %d node %lld: feature %d >= n_inputs", t, (long long)id, f);
+                const int32_t l = d->left[b + id], r = d->right[b + id];
+                if (l < 0 || l >= n || r < 0 || r >= n)
+                    return fail(SYN_ERR_INVALID_ARG, "tree %d node %lld: child id outside the tree", t, (long long)id);
+                if (seen[l] || seen[r] || l == r)
+                    return fail(SYN_ERR_INVALID_ARG, "tree %d node %lld: a node is reached twice (not a tree)", t, (long long)id);
+                seen[l] = seen[r] = 1;
+                if (qdepth[p] + 1 > SYNERGY_MAX_DEPTH)
+                    return fail(SYN_ERR_UNSUPPORTED, "tree %d deeper than %d", t, SYNERGY_MAX_DEPTH);
+                const int32_t delta = (int32_t)(queue.size() - p);
+                queue.push_back(l);
+                qdepth.push_back(qdepth[p] + 1);
+                queue.push_back(r);
+                qdepth.push_back(qdepth[p] + 1);
+                nodes.push_back(make_uint2(vb, ((uint32_t)delta << kCodeBits) | (uint32_t)f));
+            }
+            trees[t] = make_int2((int)base, depth);
+            max_depth = std::max(max_depth, depth);
+        }
+    }
+    const int pad_leaf = (int)nodes.size();
+    nodes.push_back(make_uint2(0u, 0xFFFFFF00u | leaf_code));
+
+    DeviceGuard g(device);
+    if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
+    const size_t nb = nodes.size() * sizeof(uint2);
+    const size_t tb = std::max<size_t>(trees.size(), 1) * sizeof(int2);
+    const size_t lb = (size_t)d->n_inputs * sizeof(double);
+    const size_t off_t = (nb + 255) / 256 * 256, off_l = off_t + (tb + 255) / 256 * 256;
+    const size_t total = off_l + lb;
+    void* mem = nullptr;
+    cudaError_t e = cudaMalloc(&mem, total);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(model)");
+    char* base = static_cast<char*>(mem);
+    std::vector<double> lw((size_t)d->n_inputs, 0.0);
+    if (d->linear_weight != 0.0) std::copy(d->lin_w, d->lin_w + d->n_inputs, lw.begin());
+    if ((e = cudaMemcpy(base, nodes.data(), nb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (!trees.empty() && (e = cudaMemcpy(base + off_t, trees.data(), trees.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
+        (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess) {
+        cudaFree(mem);
+        return cuda_fail(e, "cudaMemcpy(model)");
+    }
+    syn_model* m = new (std::nothrow) syn_model;
+    if (!m) {
+        cudaFree(mem);
+        return fail(SYN_ERR_OOM, "host allocation failed");
+    }
+    m->device = device;
+    m->n_inputs = d->n_inputs;
+    m->n_trees = d->forest_weight != 0.0 ? d->n_trees : 0;
+    m->max_depth = max_depth;
+    m->n_nodes = (long long)nodes.size() - 1;
+    m->bytes = (long long)total;
+    m->alloc = mem;
+    m->dm.nodes = reinterpret_cast<const uint2*>(base);
+    m->dm.trees = reinterpret_cast<const int2*>(base + off_t);
+    m->dm.lin_w = reinterpret_cast<const double*>(base + off_l);
+    m->dm.lin_b = d->linear_weight != 0.0 ? d->lin_b : 0.0;
+    m->dm.lin_weight = d->linear_weight;
+    m->dm.forest_weight = d->forest_weight;
+    m->dm.n_trees = m->n_trees;
+    m->dm.pad_leaf = pad_leaf;
+    *out = m;
+    return ok();
+}
+
+syn_status synergy_model_destroy(syn_model* m) {
+    if (!m) return ok();
+    {
+        DeviceGuard g(m->device);
+        cudaFree(m->alloc);
+    }
+    delete m;
+    return ok();
+}
+
+syn_status synergy_model_info(const syn_model* m, int32_t* n_inputs, int32_t* n_trees, int64_t* n_nodes,
+                              int32_t* max_depth, int64_t* device_bytes) {
+    if (!m) return fail(SYN_ERR_INVALID_ARG, "model is NULL");
+    if (n_inputs) *n_inputs = m->n_inputs;
+    if (n_trees) *n_trees = m->n_trees;
+    if (n_nodes) *n_nodes = m->n_nodes;
+    if (max_depth) *max_depth = m->max_depth;
+    if (device_bytes) *device_bytes = m->bytes;
+    return ok();
+}
+
+syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, syn_clocks** out) {
+    if (!out) return fail(SYN_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (!h) return fail(SYN_ERR_INVALID_ARG, "h_freqs is NULL");
+    if (n_f < 1 || n_f > SYNERGY_MAX_FREQS) return fail(SYN_ERR_INVALID_ARG, "n_freqs=%d outside [1, %d]", n_f, SYNERGY_MAX_FREQS);
+    for (int i = 0; i < n_f; ++i)
+        if (!std::isfinite(h[i])) return fail(SYN_ERR_INVALID_ARG, "freqs[%d] is not finite", i);
+    for (int i = 1; i < n_f; ++i)
+        if (!(h[i - 1] < h[i])) return fail(SYN_ERR_INVALID_ARG, "freqs not strictly ascending at %d", i);
+    DeviceGuard g(device);
+    if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
+    float* d = nullptr;
+    cudaError_t e = cudaMalloc(&d, (size_t)n_f * sizeof(float));
+    if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(clocks)");
+    if ((e = cudaMemcpy(d, h, (size_t)n_f * sizeof(float), cudaMemcpyHostToDevice)) != cudaSuccess) {
+        cudaFree(d);
+        return cuda_fail(e, "cudaMemcpy(clocks)");
+    }
+    syn_clocks* c = new (std::nothrow) syn_clocks;
+    if (!c) {
+        cudaFree(d);
+        return fail(SYN_ERR_OOM, "host allocation failed");
+    }
+    c->device = device;
+    c->n_f = n_f;
+    c->d_freqs = d;
+    *out = c;
+    return ok();
+}
+
+syn_status synergy_clocks_destroy(syn_clocks* c) {
+    if (!c) return ok();
+    {
+        DeviceGuard g(c->device);
+        cudaFree(c->d_freqs);
+    }
+    delete c;
+    return ok();
+}
+
+syn_status synergy_clocks_info(const syn_clocks* c, int32_t* n_freqs) {
+    if (!c) return fail(SYN_ERR_INVALID_ARG, "clocks is NULL");
+    if (n_freqs) *n_freqs = c->n_f;
+    return ok();
+}
+
+syn_status synergy_predict(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
+                           int32_t F, const syn_clocks* clocks, int32_t def, float* d_S, float* d_E,
+                           syn_stream stream) {
+    return run_sweep(sp, en, d_features, n_k, F, clocks, def, nullptr, 0, nullptr, d_S, d_E, kModePredict,
+                     static_cast<cudaStream_t>(stream));
+}
+
+syn_status synergy_sweep(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
+                         int32_t F, const syn_clocks* clocks, int32_t def, const syn_target* targets,
+                         int32_t n_t, int32_t* d_choice, float* d_S, float* d_E, syn_stream stream) {
+    return run_sweep(sp, en, d_features, n_k, F, clocks, def, targets, n_t, d_choice, d_S, d_E, kModeSweep,
+                     static_cast<cudaStream_t>(stream));
+}
+
+syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32_t n_f, int32_t def,
+                          const syn_target* targets, int32_t n_t, int32_t* d_choice, syn_stream stream) {
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    if (n_f < 1 || n_f > SYNERGY_MAX_FREQS) return fail(SYN_ERR_INVALID_ARG, "n_freqs=%d outside [1, %d]", n_f, SYNERGY_MAX_FREQS);
+    if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
+    syn_status s = check_targets(targets, n_t);
+    if (s != SYN_OK) return s;
+    if (n_k == 0) {
+        g_last = {0, 0, 0, 0, 0};
+        return ok();
+    }
+    if (!d_S || !d_E || !d_choice) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    SelectArgs a;
+    memset(&a, 0, sizeof a);
+    a.S = d_S;
+    a.E = d_E;
+    a.n_k = n_k;
+    a.n_f = n_f;
+    a.def = def;
+    a.n_t = n_t;
+    for (int t = 0; t < n_t; ++t) {
+        a.kind[t] = targets[t].kind;
+        a.x[t] = targets[t].x;
+    }
+    a.choice = d_choice;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const int block = 256;
+    const long long need = (n_k + 7) / 8;
+    const long long grid = std::min<long long>(need, (long long)sm_count(dev) * 8);
+    k_select<<<(unsigned)grid, block, 0, static_cast<cudaStream_t>(stream)>>>(a);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "k_select launch");
+    g_last = {1, n_k * (long long)n_f, grid, block, 0};
+    return ok();
+}
+
+syn_status synergy_workspace_create(int32_t device, syn_workspace** out) {
+    if (!out) return fail(SYN_ERR_INVALID_ARG, "out is NULL");
+    syn_workspace* w = new (std::nothrow) syn_workspace;
+    if (!w) return fail(SYN_ERR_OOM, "host allocation failed");
+    w->device = device;
+    w->d_features = nullptr;
+    w->cap_features = 0;
+    w->d_choice = nullptr;
+    w->cap_choice = 0;
+    *out = w;
+    return ok();
+}
+
+syn_status synergy_workspace_destroy(syn_workspace* w) {
+    if (!w) return ok();
+    {
+        DeviceGuard g(w->device);
+        cudaFree(w->d_features);
+        cudaFree(w->d_choice);
+    }
+    delete w;
+    return ok();
+}
+
+syn_status synergy_sweep_host(syn_workspace* w, const syn_model* sp, const syn_model* en, const float* h_features,
+                              int64_t n_k, int32_t F, const syn_clocks* clocks, int32_t def,
+                              const syn_target* targets, int32_t n_t, int32_t* h_choice, syn_stream stream) {
+    if (!w) return fail(SYN_ERR_INVALID_ARG, "workspace is NULL");
+    if (!clocks || !current_device_is(w->device) || clocks->device != w->device)
+        return fail(SYN_ERR_INVALID_ARG, "workspace/clocks device differs from the current device");
+    if (n_k > 0 && (!h_features || !h_choice)) return fail(SYN_ERR_INVALID_ARG, "host buffer is NULL");
+    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, kModeSweep);
+    if (vs != SYN_OK) return vs;
+    const size_t fb = (size_t)n_k * (size_t)F * sizeof(float);
+    const size_t cb = (size_t)n_k * (size_t)std::max(n_t, 0) * sizeof(int32_t);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaError_t e;
+    if (fb > w->cap_features) {
+        cudaFree(w->d_features);
+        w->d_features = nullptr;
+        w->cap_features = 0;
+        if ((e = cudaMalloc(&w->d_features, fb)) != cudaSuccess) return cuda_fail(e, "cudaMalloc(workspace)");
+        w->cap_features = fb;
+    }
+    if (cb > w->cap_choice) {
+        cudaFree(w->d_choice);
+        w->d_choice = nullptr;
+        w->cap_choice = 0;
+        if ((e = cudaMalloc(&w->d_choice, cb)) != cudaSuccess) return cuda_fail(e, "cudaMalloc(workspace)");
+        w->cap_choice = cb;
+    }
+    if (n_k > 0 && (e = cudaMemcpyAsync(w->d_features, h_features, fb, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+        return cuda_fail(e, "cudaMemcpyAsync H2D");
+    syn_status s = run_sweep(sp, en, w->d_features, n_k, F, clocks, def, targets, n_t, w->d_choice, nullptr,
+                             nullptr, kModeSweep, st);
+    if (s != SYN_OK) return s;
+    if (n_k > 0 && (e = cudaMemcpyAsync(h_choice, w->d_choice, cb, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
+        return cuda_fail(e, "cudaMemcpyAsync D2H");
+    return ok();
+}
+
+syn_status synergy_last_launch(int32_t* kernels, int64_t* evals, int64_t* grid, int32_t* block, int32_t* variant) {
+    if (kernels) *kernels = g_last.kernels;
+    if (evals) *evals = g_last.evals;
+    if (grid) *grid = g_last.grid;
+    if (block) *block = g_last.block;
+    if (variant) *variant = g_last.variant;
+    return ok();
+}
+
+}  // extern "C"

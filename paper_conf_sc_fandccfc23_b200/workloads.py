@@ -150,7 +150,7 @@ def _feature_chunk(seed_seq: np.random.SeedSequence, chunk: int, rows: int, F: i
 
 
 def gen_features(seed_seq, n_rows: int, F: int, row0: int = 0, n: Optional[int] = None) -> np.ndarray:
-    """Rows [row0, row0+n) of the (conceptually n_rows-long) feature table.
+    """Rows [row0, row0+n) of an unbounded seeded feature population (n defaults to n_rows-row0).
 
     Values floor(2^U(0,10)) (integer counts 1..1023, exact in fp32), zeros with prob 0.25
     for often-absent op classes else 0.05.  Chunked so any shard regenerates alone.
@@ -162,7 +162,7 @@ def gen_features(seed_seq, n_rows: int, F: int, row0: int = 0, n: Optional[int] 
     while r < row0 + n:
         c = r // FEATURE_CHUNK
         c0 = c * FEATURE_CHUNK
-        rows = min(FEATURE_CHUNK, n_rows - c0)
+        rows = FEATURE_CHUNK          # chunk contents never depend on n_rows
         blk = _feature_chunk(seed_seq, c, rows, F)
         a = r - c0
         b = min(rows, row0 + n - c0)

@@ -1,0 +1,158 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Bar (north_star): predictions fp32 within 1e-5 relative — asserted here
+bit-exact because both sides run the identical fp64 op sequence; choices bit-exact (the
+tolerance exemption for near-tied objectives is counted and must be 0).
+"""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_fandccfc23_b200 import workloads as W
+from gpu_util import assert_bits_equal, assert_choices, gpu_models, gpu_predict, gpu_sweep
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _build():
+    from paper_conf_sc_fandccfc23_b200 import build
+    build.build()
+    oracle.build()
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c2"])
+def test_full_config_bit_exact(cfg):
+    w = W.make_config(cfg)
+    ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
+    got = gpu_sweep(w, want_pred=True)
+    assert_bits_equal(got["S"], ref["S"], "S")
+    assert_bits_equal(got["E"], ref["E"], "E")
+    assert_choices(got["choice"], ref["choice"], ref["gap"])
+
+
+def test_predict_matches_sweep_predictions_and_raw_mode():
+    w = W.make_config("c1")
+    S, E = gpu_predict(w)
+    rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, w.default_idx)
+    assert_bits_equal(S, rS, "S")
+    assert_bits_equal(E, rE, "E")
+    S, E = gpu_predict(w, default_idx=-1)
+    rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
+    assert_bits_equal(S, rS, "raw S")
+    assert_bits_equal(E, rE, "raw E")
+
+
+FUZZ = [
+    # (n_kernels, n_freqs, F, n_trees, max_depth, linear, extra)
+    (1, 1, 3, 2, 3, "none", {}),
+    (3, 2, 4, 3, 4, "none", {}),
+    (7, 31, 5, 4, 6, "none", {"exact_thresholds": True}),
+    (9, 32, 5, 5, 6, "none", {"exact_thresholds": True}),
+    (13, 33, 6, 1, 8, "none", {}),
+    (17, 64, 12, 7, 10, "none", {"p_leaf": 0.05}),
+    (5, 196, 12, 9, 12, "none", {"p_leaf": 0.3}),
+    (11, 97, 7, 3, 5, "only", {}),
+    (11, 97, 7, 6, 5, "both", {}),
+    (2, 600, 4, 3, 9, "none", {}),
+    (1, 4096, 3, 2, 7, "none", {}),
+    (300, 128, 12, 3, 6, "none", {}),
+    (1100, 40, 6, 2, 4, "none", {"value_range": (-0.5, 1.5)}),        # non-positive predictions
+    (40, 50, 6, 2, 0, "none", {}),                                    # depth-0 stumps: constant
+]
+
+
+@pytest.mark.parametrize("case", range(len(FUZZ)))
+def test_fuzz_bit_exact(case):
+    n_k, n_f, F, T, D, lin, kw = FUZZ[case]
+    w = W.fuzz_workload(1000 + case, n_k, n_f, F=F, n_trees=T, max_depth=D, linear=lin, **kw)
+    targets_a, targets_b = w.targets[:8], w.targets[8:]
+    for tg in (targets_a, targets_b):
+        w.targets = tg
+        ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
+        got = gpu_sweep(w, want_pred=True)
+        assert_bits_equal(got["S"], ref["S"], "S")
+        assert_bits_equal(got["E"], ref["E"], "E")
+        assert_choices(got["choice"], ref["choice"], ref["gap"])
+
+
+def test_empty_batch_is_noop():
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.fuzz_workload(5, 0, 16)
+    sp, en, ck = gpu_models(w)
+    out = syn.sweep(sp, en, torch.empty((0, w.n_features), device="cuda"), ck, w.default_idx, w.targets[:6])
+    assert out.shape == (0, 6)
+
+
+def test_standalone_select_on_oracle_predictions_with_invalid_entries():
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    rng = np.random.default_rng(77)
+    for n_f in (1, 5, 32, 33, 196, 1000):
+        n_k = 257
+        S = rng.integers(1, 17, size=(n_k, n_f)).astype(np.float32) / 8          # exact ties
+        E = rng.integers(1, 17, size=(n_k, n_f)).astype(np.float32) / 8
+        S[rng.uniform(size=S.shape) < 0.05] = 0.0
+        E[rng.uniform(size=E.shape) < 0.05] = np.nan
+        S[rng.uniform(size=S.shape) < 0.02] = np.inf
+        d = int(rng.integers(0, n_f))
+        targets = W.targets_six() + [(W.ES, 100.0), (W.PL, 0.0), (W.ES, 33.0), (W.PL, 100.0)]
+        ref = oracle.select(S, E, d, targets)
+        got = syn.select(torch.from_numpy(S).cuda(), torch.from_numpy(E).cuda(), d, targets).cpu().numpy()
+        assert_choices(got, ref)
+
+
+def test_host_buffer_path_matches_device_path():
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.make_config("c1")
+    sp, en, ck = gpu_models(w)
+    ws = syn.Workspace(0)
+    hf = torch.from_numpy(w.features.copy()).pin_memory()
+    ho = torch.empty((w.n_kernels, len(w.targets)), dtype=torch.int32).pin_memory()
+    ws.sweep_host(sp, en, hf, ck, w.default_idx, w.targets, ho)
+    torch.cuda.synchronize()
+    ref = oracle.sweep_workload(w)
+    assert_choices(ho.numpy(), ref["choice"])
+
+
+def test_invalid_arguments_enqueue_nothing():
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.make_config("c1")
+    sp, en, ck = gpu_models(w)
+    feats = torch.from_numpy(w.features).cuda()
+    out = torch.full((w.n_kernels, 6), 12345, dtype=torch.int32, device="cuda")
+    with pytest.raises(syn.SynergyError) as ei:
+        syn.sweep(sp, en, feats, ck, w.n_freqs, w.targets, out=out)            # default out of range
+    assert ei.value.status == syn.SYN_ERR_INVALID_ARG
+    with pytest.raises(syn.SynergyError):
+        syn.sweep(sp, en, feats[:, :5].contiguous(), ck, w.default_idx, w.targets, out=out)   # F mismatch
+    with pytest.raises(syn.SynergyError):
+        syn.sweep(sp, en, feats, ck, w.default_idx, [(9, 0.0)], out=out[:, :1].contiguous())
+    torch.cuda.synchronize()
+    assert bool((out == 12345).all())
+
+
+# ------------------------------------------------- full sizes, bench launch config, sampled
+
+@pytest.mark.parametrize("cfg,n_sample", [("c3", 48), ("c4", 384), ("c5", 3584)])
+def test_full_size_sampled(cfg, n_sample):
+    """The GPU runs the whole config in the launch configuration bench.py times; the oracle
+    recomputes a seeded sample of kernel rows (c5: all rows; its 64 replicas must agree)."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.make_config(cfg)
+    sp, en, ck = gpu_models(w)
+    feats = torch.from_numpy(w.features).cuda()
+    ch = syn.sweep(sp, en, feats, ck, w.default_idx, w.targets).cpu().numpy()
+    rng = np.random.default_rng(2024)
+    rows = np.sort(rng.choice(w.n_kernels, size=min(n_sample, w.n_kernels), replace=False))
+    rows = np.unique(np.concatenate([rows, [0, w.n_kernels - 1]]))
+    ref = oracle.sweep(w.speedup, w.energy, w.features[rows], w.freqs, w.default_idx, w.targets, with_gap=True)
+    assert_choices(ch[rows], ref["choice"], ref["gap"])
+    assert (ch >= 0).all() and (ch < w.n_freqs).all()
+    if cfg == "c5":
+        blocks = ch.reshape(64, W.C5_BLOCK, -1)
+        assert (blocks == blocks[0]).all()
