@@ -288,9 +288,9 @@ def main():
         flush.zero_()
         step()
     t_end = time.time() + 0.5
-    while time.time() < t_end:
+    while time.time() < t_end:          # bounded: one step in flight at a time
         step()
-    torch.cuda.synchronize()
+        torch.cuda.synchronize()
 
     K = args.steps
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),

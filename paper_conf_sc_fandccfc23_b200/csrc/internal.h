@@ -49,6 +49,12 @@ struct SweepArgs {
     int mode;
     int tile_k;              // kernels per CTA
     int xs;                  // x-vector stride in smem (floats)
+    // clock-interval traversal (k_sweep_iv) only
+    int tc;                  // trees per chunk (one (kernel, tree) task per thread)
+    int words;               // ceil(n_f / 32) run-start mask words per task
+    int vcap;                // run values kept per task
+    int vs;                  // run-value stride per task (odd, conflict-free)
+    int region;              // bytes of the task region (also holds the float finish scratch)
 };
 
 struct SelectArgs {

@@ -153,6 +153,37 @@ __device__ __forceinline__ void select_row_warp(const float* S, const float* E, 
     }
 }
 
+// Per kernel of the tile (one warp each): normalise the raw fp64 model outputs to the default
+// clock (S = (float)(mS_i / mS_def), L69 / DESIGN.md Q13; raw (float)m when def == -1), write
+// the predictions if requested, then run the per-target selection.  mS/mE: [nk][n_f] doubles,
+// sS/sE: [nk][n_f] float scratch, all in shared memory.  Caller has synchronised the block.
+__device__ __forceinline__ void finish_tile(const SweepArgs& a, const double* mS, const double* mE,
+                                            float* sS, float* sE, int nk, long long k0) {
+    const int n_f = a.n_f;
+    const int lane = threadIdx.x & 31;
+    const int nw = blockDim.x >> 5;
+    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
+        const double* rS = mS + (size_t)kl * n_f;
+        const double* rE = mE + (size_t)kl * n_f;
+        float* oS = sS + (size_t)kl * n_f;
+        float* oE = sE + (size_t)kl * n_f;
+        const long long k = k0 + kl;
+        const double dS = a.def >= 0 ? rS[a.def] : 1.0;
+        const double dE = a.def >= 0 ? rE[a.def] : 1.0;
+        for (int i = lane; i < n_f; i += 32) {
+            const float s = a.def >= 0 ? __double2float_rn(__ddiv_rn(rS[i], dS)) : __double2float_rn(rS[i]);
+            const float e = a.def >= 0 ? __double2float_rn(__ddiv_rn(rE[i], dE)) : __double2float_rn(rE[i]);
+            oS[i] = s;
+            oE[i] = e;
+            if (a.S_out) a.S_out[k * n_f + i] = s;
+            if (a.E_out) a.E_out[k * n_f + i] = e;
+        }
+        __syncwarp();
+        if (a.mode == kModeSweep)
+            select_row_warp(oS, oE, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
+    }
+}
+
 template <int SLOTS, int TILP>
 __global__ void __launch_bounds__(512) k_sweep(const __grid_constant__ SweepArgs a) {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -206,29 +237,7 @@ __global__ void __launch_bounds__(512) k_sweep(const __grid_constant__ SweepArgs
     }
     __syncthreads();
 
-    // phase 2: per kernel (one warp each): normalise to the default clock, then select
-    const int lane = threadIdx.x & 31;
-    const int nw = blockDim.x >> 5;
-    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
-        const double* rS = mS + (size_t)kl * n_f;
-        const double* rE = mE + (size_t)kl * n_f;
-        float* oS = sS + (size_t)kl * n_f;
-        float* oE = sE + (size_t)kl * n_f;
-        const long long k = k0 + kl;
-        const double dS = a.def >= 0 ? rS[a.def] : 1.0;
-        const double dE = a.def >= 0 ? rE[a.def] : 1.0;
-        for (int i = lane; i < n_f; i += 32) {
-            const float s = a.def >= 0 ? __double2float_rn(__ddiv_rn(rS[i], dS)) : __double2float_rn(rS[i]);
-            const float e = a.def >= 0 ? __double2float_rn(__ddiv_rn(rE[i], dE)) : __double2float_rn(rE[i]);
-            oS[i] = s;
-            oE[i] = e;
-            if (a.S_out) a.S_out[k * n_f + i] = s;
-            if (a.E_out) a.E_out[k * n_f + i] = e;
-        }
-        __syncwarp();
-        if (a.mode == kModeSweep)
-            select_row_warp(oS, oE, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
-    }
+    finish_tile(a, mS, mE, sS, sE, nk, k0);
 }
 
 // Standalone selection: one warp per kernel row, rows read from HBM (L1-resident across the

@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -13,6 +14,7 @@
 
 #include "internal.h"
 #include "kernels.cuh"
+#include "kernels_iv.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -115,9 +117,16 @@ syn_status check_targets(const syn_target* t, int32_t n_t) {
 // ---------------------------------------------------------------- launch configuration
 
 struct Config {
+    int algo;                 // 0 = direct traversal (k_sweep), 1 = clock-interval (k_sweep_iv)
     int slots, tilp, tile_k, nt, xs;
+    int tc, words, vcap, vs, region;
     size_t smem;
 };
+
+int env_int(const char* name, int dflt) {
+    const char* v = getenv(name);
+    return (v && *v) ? atoi(v) : dflt;
+}
 
 size_t sweep_smem(int tile_k, int n_f, int xs) {
     return (size_t)tile_k * ((size_t)n_f * 24 + (size_t)xs * 4) + (size_t)n_f * 4;
@@ -127,6 +136,8 @@ size_t sweep_smem(int tile_k, int n_f, int xs) {
 // SM busy for small batches (slots=1, 4 trees in flight) and amortises staging for large ones.
 Config choose_config(long long n_k, int n_f, int F, int dev) {
     Config c;
+    c.algo = 0;
+    c.tc = c.words = c.vcap = c.vs = c.region = 0;
     const long long resident = (long long)sm_count(dev) * 2048;
     const long long evals = n_k * (long long)n_f;
     c.slots = evals >= 16 * resident ? 8 : evals >= 8 * resident ? 4 : evals >= 4 * resident ? 2 : 1;
@@ -141,6 +152,55 @@ Config choose_config(long long n_k, int n_f, int F, int dev) {
     c.nt = (int)std::min<long long>(std::max<long long>(thr, 32), 512);
     c.smem = sweep_smem(c.tile_k, n_f, c.xs);
     return c;
+}
+
+// Clock-interval kernel: NT threads, TK kernels per CTA, TC = NT / TK trees per chunk (one
+// (kernel, tree) task per thread), accumulators for the TK x n_f units in shared memory.
+// Small batches use TK = 1 so the grid spans the SMs; large ones TK = 4 so a chunk's trees are
+// shared by more kernels (L1 reuse of the upper levels).
+size_t iv_smem(int nt, int tk, int n_f, int xs, int words, int vs, int* region) {
+    const int tc = std::max(1, nt / tk);
+    size_t tasks = (size_t)tc * tk * ((size_t)words * 8 + (size_t)vs * 8);
+    tasks = std::max(tasks, (size_t)tk * n_f * 8);            // finish-phase float scratch
+    tasks = (tasks + 15) & ~(size_t)15;
+    *region = (int)tasks;
+    return (size_t)tk * n_f * 16 + tasks + (size_t)n_f * 4 + (size_t)tk * xs * 4 + (kGrid + 1) * 2 + 16;
+}
+
+bool choose_iv(long long n_k, int n_f, int F, int dev, Config& c) {
+    if (n_f > 1024) return false;
+    const int sms = sm_count(dev);
+    c.nt = env_int("SYNERGY_NT", 128) >= 256 ? 256 : 128;
+    int tk = (int)std::min<long long>(4, std::max<long long>(1, n_k / (8LL * sms)));
+    tk = env_int("SYNERGY_TK", tk);
+    tk = (int)std::max<long long>(1, std::min<long long>(std::min(tk, c.nt), std::max<long long>(n_k, 1)));
+    c.algo = 1;
+    c.slots = 0;
+    c.tilp = 0;
+    c.tile_k = tk;
+    c.xs = (F + 2) | 1;
+    c.tc = std::max(1, c.nt / tk);
+    c.words = (n_f + 31) / 32;
+    c.vcap = std::max(1, env_int("SYNERGY_VCAP", 24));
+    c.vs = c.vcap | 1;
+    c.smem = iv_smem(c.nt, tk, n_f, c.xs, c.words, c.vs, &c.region);
+    return c.smem <= 220 * 1024;
+}
+
+template <int NT, int MINB>
+cudaError_t launch_iv_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    static size_t smem_set = 48 * 1024;
+    if (c.smem > smem_set) {
+        cudaError_t e = cudaFuncSetAttribute(k_sweep_iv<NT, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        if (e != cudaSuccess) return e;
+        smem_set = c.smem;
+    }
+    k_sweep_iv<NT, MINB><<<(unsigned)grid, NT, c.smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_iv(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    return c.nt == 256 ? launch_iv_t<256, 4>(a, c, grid, st) : launch_iv_t<128, 8>(a, c, grid, st);
 }
 
 template <int S, int T>
@@ -217,14 +277,26 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     a.S_out = d_S;
     a.E_out = d_E;
     a.mode = mode;
-    const Config c = choose_config(n_k, n_f, F, clocks->device);
+    // default: clock-interval traversal when forests are present and n_f <= 1024;
+    // SYNERGY_ALGO=direct forces the per-clock root-to-leaf kernel (A/B and fallback)
+    const char* algo_env = getenv("SYNERGY_ALGO");
+    const bool force_direct = algo_env && !strcmp(algo_env, "direct");
+    Config c;
+    const bool forests = sp->n_trees > 0 || en->n_trees > 0;
+    if (force_direct || !forests || !choose_iv(n_k, n_f, F, clocks->device, c))
+        c = choose_config(n_k, n_f, F, clocks->device);
     a.tile_k = c.tile_k;
     a.xs = c.xs;
+    a.tc = c.tc;
+    a.words = c.words;
+    a.vcap = c.vcap;
+    a.vs = c.vs;
+    a.region = c.region;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    cudaError_t e = launch_sweep(a, c, grid, st);
-    if (e != cudaSuccess) return cuda_fail(e, "k_sweep launch");
-    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.slots * 10 + c.tilp};
+    cudaError_t e = c.algo == 1 ? launch_iv(a, c, grid, st) : launch_sweep(a, c, grid, st);
+    if (e != cudaSuccess) return cuda_fail(e, c.algo == 1 ? "k_sweep_iv launch" : "k_sweep launch");
+    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.algo ? 1000 + c.tile_k : c.slots * 10 + c.tilp};
     return ok();
 }
 

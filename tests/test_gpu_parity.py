@@ -21,8 +21,28 @@ def _build():
     oracle.build()
 
 
+# Kernel variants the library can pick (read per call from the environment):
+#   default   clock-interval traversal (k_sweep_iv), auto tile
+#   direct    per-clock root-to-leaf traversal (k_sweep)
+#   vcap1     interval kernel keeping only 1 run value per (kernel, tree): exercises the
+#             direct-walk fallback for every later run
+#   tk3       interval kernel with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
+#   nt256tk5  interval kernel, 256 threads, 5 kernels per CTA (51 trees per chunk)
+VARIANTS = {"default": {}, "direct": {"SYNERGY_ALGO": "direct"}, "vcap1": {"SYNERGY_VCAP": "1"},
+            "tk3": {"SYNERGY_TK": "3"}, "nt256tk5": {"SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
+
+
+@pytest.fixture(params=list(VARIANTS))
+def variant(request, monkeypatch):
+    for k in ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT"):
+        monkeypatch.delenv(k, raising=False)
+    for k, v in VARIANTS[request.param].items():
+        monkeypatch.setenv(k, v)
+    return request.param
+
+
 @pytest.mark.parametrize("cfg", ["c1", "c2"])
-def test_full_config_bit_exact(cfg):
+def test_full_config_bit_exact(cfg, variant):
     w = W.make_config(cfg)
     ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
     got = gpu_sweep(w, want_pred=True)
@@ -31,7 +51,7 @@ def test_full_config_bit_exact(cfg):
     assert_choices(got["choice"], ref["choice"], ref["gap"])
 
 
-def test_predict_matches_sweep_predictions_and_raw_mode():
+def test_predict_matches_sweep_predictions_and_raw_mode(variant):
     w = W.make_config("c1")
     S, E = gpu_predict(w)
     rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, w.default_idx)
@@ -63,7 +83,7 @@ FUZZ = [
 
 
 @pytest.mark.parametrize("case", range(len(FUZZ)))
-def test_fuzz_bit_exact(case):
+def test_fuzz_bit_exact(case, variant):
     n_k, n_f, F, T, D, lin, kw = FUZZ[case]
     w = W.fuzz_workload(1000 + case, n_k, n_f, F=F, n_trees=T, max_depth=D, linear=lin, **kw)
     targets_a, targets_b = w.targets[:8], w.targets[8:]
