@@ -26,6 +26,17 @@ struct DevModel {
     double forest_weight;    // 0 => absent
     int n_trees;
     int pad_leaf;            // index of the padding leaf
+    int depth;               // deepest root-to-leaf path over all trees (edges)
+    // 2-level block layout (32 B per block, two uint4): words
+    //   0: thr(n)  1: thr(c0)  2: thr(c1)  3: code(n) | code(c0) << 8 | code(c1) << 16 |
+    //                                         leafmask << 24 (grandchild slot holds a leaf value)
+    //   4..7: grandchild slots g = 2*d0 + d1: block index, or fp32 leaf-value bits (leafmask)
+    // A child c_d that is itself a leaf has code F+1 and its value in thr(c_d); a one-leaf tree
+    // has code(n) = F+1.  Blocks exist for the root and every internal node at even depth, so
+    // a root-to-leaf walk of depth D takes max(1, ceil(D / 2)) block loads.
+    const uint4* blocks;
+    const int* broot;        // [n_trees] root block of each tree
+    int bdepth;              // max(1, ceil(depth / 2)) over all trees
 };
 
 constexpr int kMaxTargets = 16;
@@ -55,6 +66,10 @@ struct SweepArgs {
     int vcap;                // run values kept per task
     int vs;                  // run-value stride per task (odd, conflict-free)
     int region;              // bytes of the task region (also holds the float finish scratch)
+    // warp-streaming (k_sweep_ws) only
+    int win;                 // ring-window slots per warp
+    int slot_bytes;          // bytes per slot
+    int head_bytes;          // bytes of the staged clocks / features / grid head
 };
 
 struct SelectArgs {

@@ -15,6 +15,7 @@
 #include "internal.h"
 #include "kernels.cuh"
 #include "kernels_iv.cuh"
+#include "kernels_ws.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -120,6 +121,7 @@ struct Config {
     int algo;                 // 0 = direct traversal (k_sweep), 1 = clock-interval (k_sweep_iv)
     int slots, tilp, tile_k, nt, xs;
     int tc, words, vcap, vs, region;
+    int win, slot_bytes, head_bytes;
     size_t smem;
 };
 
@@ -138,6 +140,7 @@ Config choose_config(long long n_k, int n_f, int F, int dev) {
     Config c;
     c.algo = 0;
     c.tc = c.words = c.vcap = c.vs = c.region = 0;
+    c.win = c.slot_bytes = c.head_bytes = 0;
     const long long resident = (long long)sm_count(dev) * 2048;
     const long long evals = n_k * (long long)n_f;
     c.slots = evals >= 16 * resident ? 8 : evals >= 8 * resident ? 4 : evals >= 4 * resident ? 2 : 1;
@@ -201,6 +204,53 @@ cudaError_t launch_iv_t(const SweepArgs& a, const Config& c, long long grid, cud
 
 cudaError_t launch_iv(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
     return c.nt == 256 ? launch_iv_t<256, 4>(a, c, grid, st) : launch_iv_t<128, 8>(a, c, grid, st);
+}
+
+// Warp-streaming kernel: KPC kernels per CTA, one warp per (kernel, model), WIN-slot ring
+// window of finished trees per warp, accumulators in registers (n_f <= 256).
+bool choose_ws(long long n_k, int n_f, int F, int dev, Config& c) {
+    if (n_f > 256) return false;
+    int kpc = env_int("SYNERGY_KPC", 2);
+    kpc = std::max(1, std::min(kpc, 4));
+    kpc = (int)std::min<long long>(kpc, std::max<long long>(n_k, 1));
+    c.algo = 2;
+    c.slots = 0;
+    c.tilp = 0;
+    c.tile_k = kpc;
+    c.nt = 64 * kpc;
+    c.xs = (F + 2) | 1;
+    c.words = (n_f + 31) / 32;
+    c.vcap = std::max(1, env_int("SYNERGY_VCAP", 32));
+    c.vs = c.vcap;
+    int win = std::max(32, std::min(1024, env_int("SYNERGY_WIN", 64)));
+    c.win = 32;
+    while (c.win * 2 <= win) c.win *= 2;                 // power of two: slot = tree & (WIN-1)
+    int sb = c.vs * 4 + c.words * 4 + 8;
+    c.slot_bytes = (sb + 7) & ~7;
+    c.head_bytes = (int)((((size_t)(n_f + kpc * c.xs) * 4 + (kGrid + 1) * 2) + 15) & ~(size_t)15);
+    const size_t slots = (size_t)2 * kpc * c.win * c.slot_bytes;
+    const size_t fin = (size_t)kpc * n_f * 24;
+    c.smem = c.head_bytes + std::max(slots, fin);
+    c.tc = c.region = 0;
+    return c.smem <= 220 * 1024;
+}
+
+template <int CL>
+cudaError_t launch_ws_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    static size_t smem_set = 48 * 1024;
+    if (c.smem > smem_set) {
+        cudaError_t e = cudaFuncSetAttribute(k_sweep_ws<CL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        if (e != cudaSuccess) return e;
+        smem_set = c.smem;
+    }
+    k_sweep_ws<CL><<<(unsigned)grid, c.nt, c.smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    if (c.words <= 2) return launch_ws_t<2>(a, c, grid, st);
+    if (c.words <= 4) return launch_ws_t<4>(a, c, grid, st);
+    return launch_ws_t<8>(a, c, grid, st);
 }
 
 template <int S, int T>
@@ -281,10 +331,17 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     // SYNERGY_ALGO=direct forces the per-clock root-to-leaf kernel (A/B and fallback)
     const char* algo_env = getenv("SYNERGY_ALGO");
     const bool force_direct = algo_env && !strcmp(algo_env, "direct");
+    const bool force_iv = algo_env && !strcmp(algo_env, "iv");
     Config c;
     const bool forests = sp->n_trees > 0 || en->n_trees > 0;
-    if (force_direct || !forests || !choose_iv(n_k, n_f, F, clocks->device, c))
-        c = choose_config(n_k, n_f, F, clocks->device);
+    // default: warp-streaming clock-interval kernel (n_f <= 256), else the chunked interval
+    // kernel (n_f <= 1024), else per-clock direct traversal; SYNERGY_ALGO=iv|direct forces
+    bool chosen = false;
+    if (!force_direct && forests) {
+        if (!force_iv) chosen = choose_ws(n_k, n_f, F, clocks->device, c);
+        if (!chosen) chosen = choose_iv(n_k, n_f, F, clocks->device, c);
+    }
+    if (!chosen) c = choose_config(n_k, n_f, F, clocks->device);
     a.tile_k = c.tile_k;
     a.xs = c.xs;
     a.tc = c.tc;
@@ -292,11 +349,16 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     a.vcap = c.vcap;
     a.vs = c.vs;
     a.region = c.region;
+    a.win = c.win;
+    a.slot_bytes = c.slot_bytes;
+    a.head_bytes = c.head_bytes;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    cudaError_t e = c.algo == 1 ? launch_iv(a, c, grid, st) : launch_sweep(a, c, grid, st);
-    if (e != cudaSuccess) return cuda_fail(e, c.algo == 1 ? "k_sweep_iv launch" : "k_sweep launch");
-    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.algo ? 1000 + c.tile_k : c.slots * 10 + c.tilp};
+    cudaError_t e = c.algo == 2 ? launch_ws(a, c, grid, st) : c.algo == 1 ? launch_iv(a, c, grid, st)
+                                                                         : launch_sweep(a, c, grid, st);
+    static const char* names[3] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch"};
+    if (e != cudaSuccess) return cuda_fail(e, names[c.algo]);
+    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
     return ok();
 }
 
@@ -381,13 +443,73 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     const int pad_leaf = (int)nodes.size();
     nodes.push_back(make_uint2(0u, 0xFFFFFF00u | leaf_code));
 
+    // 2-level blocks (see internal.h): built from the validated description, breadth-first
+    std::vector<uint4> blocks;
+    std::vector<int> broot;
+    int bdepth = 1;
+    if (d->forest_weight != 0.0) {
+        broot.resize(d->n_trees);
+        std::vector<int64_t> q;
+        std::vector<int64_t> qb;
+        for (int t = 0; t < d->n_trees; ++t) {
+            const int64_t b = d->tree_offset[t];
+            auto is_leaf = [&](int64_t id) { return d->feature[b + id] < 0; };
+            auto fbits = [&](int64_t id) { uint32_t u; memcpy(&u, &d->value[b + id], 4); return u; };
+            if ((blocks.size() >> 1) + 1 > 0x7ffffff0ULL) return fail(SYN_ERR_UNSUPPORTED, "too many blocks");
+            broot[t] = (int)(blocks.size() >> 1);
+            blocks.resize(blocks.size() + 2);
+            q.assign(1, 0);
+            qb.assign(1, broot[t]);
+            for (size_t p = 0; p < q.size(); ++p) {
+                const int64_t id = q[p];
+                uint32_t w[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                w[0] = fbits(id);
+                if (is_leaf(id)) {
+                    w[3] = leaf_code | (leaf_code << 8) | (leaf_code << 16);
+                } else {
+                    uint32_t codes = (uint32_t)d->feature[b + id];
+                    for (int dd = 0; dd < 2; ++dd) {
+                        const int64_t c = dd ? d->right[b + id] : d->left[b + id];
+                        w[1 + dd] = fbits(c);
+                        if (is_leaf(c)) {
+                            codes |= leaf_code << (8 + 8 * dd);
+                            continue;
+                        }
+                        codes |= (uint32_t)d->feature[b + c] << (8 + 8 * dd);
+                        for (int ee = 0; ee < 2; ++ee) {
+                            const int64_t g2 = ee ? d->right[b + c] : d->left[b + c];
+                            const int slot = 2 * dd + ee;
+                            if (is_leaf(g2)) {
+                                w[4 + slot] = fbits(g2);
+                                codes |= 1u << (24 + slot);
+                            } else {
+                                const int64_t gi = (int64_t)(blocks.size() >> 1);
+                                blocks.resize(blocks.size() + 2);
+                                w[4 + slot] = (uint32_t)gi;
+                                q.push_back(g2);
+                                qb.push_back(gi);
+                            }
+                        }
+                    }
+                    w[3] = codes;
+                }
+                blocks[2 * qb[p]] = make_uint4(w[0], w[1], w[2], w[3]);
+                blocks[2 * qb[p] + 1] = make_uint4(w[4], w[5], w[6], w[7]);
+            }
+            bdepth = std::max(bdepth, (trees[t].y + 1) / 2);
+        }
+    }
+
     DeviceGuard g(device);
     if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
     const size_t nb = nodes.size() * sizeof(uint2);
     const size_t tb = std::max<size_t>(trees.size(), 1) * sizeof(int2);
     const size_t lb = (size_t)d->n_inputs * sizeof(double);
+    const size_t bb = std::max<size_t>(blocks.size(), 2) * sizeof(uint4);
+    const size_t rb = std::max<size_t>(broot.size(), 1) * sizeof(int);
     const size_t off_t = (nb + 255) / 256 * 256, off_l = off_t + (tb + 255) / 256 * 256;
-    const size_t total = off_l + lb;
+    const size_t off_b = off_l + (lb + 255) / 256 * 256, off_r = off_b + (bb + 255) / 256 * 256;
+    const size_t total = off_r + rb;
     void* mem = nullptr;
     cudaError_t e = cudaMalloc(&mem, total);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(model)");
@@ -396,7 +518,9 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     if (d->linear_weight != 0.0) std::copy(d->lin_w, d->lin_w + d->n_inputs, lw.begin());
     if ((e = cudaMemcpy(base, nodes.data(), nb, cudaMemcpyHostToDevice)) != cudaSuccess ||
         (!trees.empty() && (e = cudaMemcpy(base + off_t, trees.data(), trees.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
-        (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess) {
+        (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (!blocks.empty() && (e = cudaMemcpy(base + off_b, blocks.data(), blocks.size() * sizeof(uint4), cudaMemcpyHostToDevice)) != cudaSuccess) ||
+        (!broot.empty() && (e = cudaMemcpy(base + off_r, broot.data(), broot.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess)) {
         cudaFree(mem);
         return cuda_fail(e, "cudaMemcpy(model)");
     }
@@ -420,6 +544,10 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.forest_weight = d->forest_weight;
     m->dm.n_trees = m->n_trees;
     m->dm.pad_leaf = pad_leaf;
+    m->dm.depth = max_depth;
+    m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
+    m->dm.broot = reinterpret_cast<const int*>(base + off_r);
+    m->dm.bdepth = bdepth;
     *out = m;
     return ok();
 }

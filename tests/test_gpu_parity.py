@@ -22,19 +22,26 @@ def _build():
 
 
 # Kernel variants the library can pick (read per call from the environment):
-#   default   clock-interval traversal (k_sweep_iv), auto tile
+#   default   warp-streaming clock-interval kernel (k_sweep_ws), 2 kernels per CTA, window 48
+#   ws_tight  k_sweep_ws with window 32 (= warp width: refills wait on the oldest tree), 1 run
+#             value kept per tree (every later run takes the direct-walk fallback), 3 kernels/CTA
+#   ws_wide   k_sweep_ws with window 128, 1 kernel per CTA
 #   direct    per-clock root-to-leaf traversal (k_sweep)
-#   vcap1     interval kernel keeping only 1 run value per (kernel, tree): exercises the
-#             direct-walk fallback for every later run
-#   tk3       interval kernel with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
-#   nt256tk5  interval kernel, 256 threads, 5 kernels per CTA (51 trees per chunk)
-VARIANTS = {"default": {}, "direct": {"SYNERGY_ALGO": "direct"}, "vcap1": {"SYNERGY_VCAP": "1"},
-            "tk3": {"SYNERGY_TK": "3"}, "nt256tk5": {"SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
+#   iv        chunked clock-interval kernel (k_sweep_iv), auto tile
+#   iv_vcap1  k_sweep_iv keeping 1 run value per (kernel, tree)
+#   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
+#   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
+VARIANTS = {"default": {}, "ws_tight": {"SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"}, "ws_wide": {"SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
+            "direct": {"SYNERGY_ALGO": "direct"}, "iv": {"SYNERGY_ALGO": "iv"},
+            "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
+            "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
+            "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
+KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC")
 
 
 @pytest.fixture(params=list(VARIANTS))
 def variant(request, monkeypatch):
-    for k in ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT"):
+    for k in KNOBS:
         monkeypatch.delenv(k, raising=False)
     for k, v in VARIANTS[request.param].items():
         monkeypatch.setenv(k, v)
