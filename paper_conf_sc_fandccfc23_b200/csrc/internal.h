@@ -37,9 +37,15 @@ struct DevModel {
     const uint4* blocks;
     const int* broot;        // [n_trees] root block of each tree
     int bdepth;              // max(1, ceil(depth / 2)) over all trees
+    // exact fixed-point leaf sums (k_sweep_da): every leaf v is an integer multiple of 2^-s and
+    // n_trees * max|v| * 2^s < 2^62, so v * fx_scale is an exact int64 and sums are exact
+    int fx_ok;
+    double fx_scale;         // 2^s
+    double fx_inv;           // 2^-s
 };
 
 constexpr int kMaxTargets = 16;
+constexpr int kGrid = 1024;     // uniform bins over [f_0, f_{n-1}] for the clock-cut lookup
 
 enum Mode : int { kModePredict = 0, kModeSweep = 1 };
 
@@ -70,6 +76,9 @@ struct SweepArgs {
     int win;                 // ring-window slots per warp
     int slot_bytes;          // bytes per slot
     int head_bytes;          // bytes of the staged clocks / features / grid head
+    // clock-cut grid built once per clock table (syn_clocks)
+    const unsigned short* grid;   // [kGrid + 1]
+    float f0, inv_step;
 };
 
 struct SelectArgs {

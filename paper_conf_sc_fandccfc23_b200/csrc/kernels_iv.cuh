@@ -24,7 +24,6 @@
 namespace syn {
 
 constexpr int kMaxStack = 64;   // >= SYNERGY_MAX_DEPTH: pending right parts of ancestors
-constexpr int kGrid = 1024;     // uniform bins over [f_0, f_{n-1}) for the clock-cut lookup
 
 // Clock cut: s = #{i : f_i <= thr} for fr[lo] <= thr < fr[hi-1].  A uniform grid over the
 // clock range gives a start index (grid[b] = #{i : f_i < f_0 + b*step}); the exact position is

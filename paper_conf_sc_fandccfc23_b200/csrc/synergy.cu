@@ -16,6 +16,7 @@
 #include "kernels.cuh"
 #include "kernels_iv.cuh"
 #include "kernels_ws.cuh"
+#include "kernels_da.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -35,6 +36,8 @@ struct syn_clocks {
     int device;
     int n_f;
     float* d_freqs;
+    unsigned short* d_grid;   // clock-cut hint table, kGrid + 1 entries
+    float f0, inv_step;
 };
 
 struct syn_workspace {
@@ -253,6 +256,44 @@ cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaS
     return launch_ws_t<8>(a, c, grid, st);
 }
 
+// Difference-array kernel: one CTA per kernel, exact int64 leaf sums (needs fx_ok forests).
+bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c) {
+    if (n_f > 2048) return false;
+    if ((sp->n_trees && !sp->dm.fx_ok) || (en->n_trees && !en->dm.fx_ok)) return false;
+    const int tt = sp->n_trees + en->n_trees;
+    int nt = env_int("SYNERGY_NT", tt > 256 ? 256 : 128);
+    nt = nt >= 256 ? 256 : (nt >= 128 ? 128 : 64);
+    c.algo = 3;
+    c.slots = c.tilp = 0;
+    c.tile_k = 1;
+    c.nt = nt;
+    c.xs = (F + 2) | 1;
+    c.tc = c.words = c.vcap = c.vs = c.region = 0;
+    c.win = c.slot_bytes = c.head_bytes = 0;
+    c.smem = (size_t)2 * (n_f + 1) * 8 + (size_t)n_f * 24 + (size_t)n_f * 4 + (size_t)c.xs * 4 +
+             (size_t)((kGrid + 2) & ~1) * 2 + 16;
+    (void)n_k;
+    return c.smem <= 220 * 1024;
+}
+
+template <int NT>
+cudaError_t launch_da_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    static size_t smem_set = 48 * 1024;
+    if (c.smem > smem_set) {
+        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        if (e != cudaSuccess) return e;
+        smem_set = c.smem;
+    }
+    k_sweep_da<NT><<<(unsigned)grid, NT, c.smem, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
+    if (c.nt == 256) return launch_da_t<256>(a, c, grid, st);
+    if (c.nt == 128) return launch_da_t<128>(a, c, grid, st);
+    return launch_da_t<64>(a, c, grid, st);
+}
+
 template <int S, int T>
 cudaError_t launch_sweep_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
     static size_t smem_set = 48 * 1024;   // per-instantiation opt-in high-water mark
@@ -332,13 +373,16 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     const char* algo_env = getenv("SYNERGY_ALGO");
     const bool force_direct = algo_env && !strcmp(algo_env, "direct");
     const bool force_iv = algo_env && !strcmp(algo_env, "iv");
+    const bool force_ws = algo_env && !strcmp(algo_env, "ws");
     Config c;
     const bool forests = sp->n_trees > 0 || en->n_trees > 0;
-    // default: warp-streaming clock-interval kernel (n_f <= 256), else the chunked interval
-    // kernel (n_f <= 1024), else per-clock direct traversal; SYNERGY_ALGO=iv|direct forces
+    // default: order-free difference-array kernel (exact int64 leaf sums; n_f <= 2048), else the
+    // in-order warp-streaming kernel (n_f <= 256), else the chunked interval kernel
+    // (n_f <= 1024), else per-clock direct traversal; SYNERGY_ALGO=ws|iv|direct forces one
     bool chosen = false;
     if (!force_direct && forests) {
-        if (!force_iv) chosen = choose_ws(n_k, n_f, F, clocks->device, c);
+        if (!force_iv && !force_ws) chosen = choose_da(sp, en, n_k, n_f, F, c);
+        if (!chosen && !force_iv) chosen = choose_ws(n_k, n_f, F, clocks->device, c);
         if (!chosen) chosen = choose_iv(n_k, n_f, F, clocks->device, c);
     }
     if (!chosen) c = choose_config(n_k, n_f, F, clocks->device);
@@ -352,11 +396,16 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     a.win = c.win;
     a.slot_bytes = c.slot_bytes;
     a.head_bytes = c.head_bytes;
+    a.grid = clocks->d_grid;
+    a.f0 = clocks->f0;
+    a.inv_step = clocks->inv_step;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    cudaError_t e = c.algo == 2 ? launch_ws(a, c, grid, st) : c.algo == 1 ? launch_iv(a, c, grid, st)
-                                                                         : launch_sweep(a, c, grid, st);
-    static const char* names[3] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch"};
+    cudaError_t e = c.algo == 3 ? launch_da(a, c, grid, st)
+                  : c.algo == 2 ? launch_ws(a, c, grid, st)
+                  : c.algo == 1 ? launch_iv(a, c, grid, st)
+                                : launch_sweep(a, c, grid, st);
+    static const char* names[4] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch", "k_sweep_da launch"};
     if (e != cudaSuccess) return cuda_fail(e, names[c.algo]);
     g_last = {1, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
     return ok();
@@ -438,6 +487,32 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
             }
             trees[t] = make_int2((int)base, depth);
             max_depth = std::max(max_depth, depth);
+        }
+    }
+    // exact fixed-point scale for the leaf sums (k_sweep_da): s = -(smallest leaf ulp exponent)
+    int fx_ok = 0, fx_s = 0;
+    if (d->forest_weight != 0.0) {
+        int min_lsb = 1 << 30, max_e = -(1 << 30);
+        bool finite = true;
+        for (int t = 0; t < d->n_trees && finite; ++t)
+            for (int64_t id = d->tree_offset[t]; id < d->tree_offset[t + 1]; ++id) {
+                if (d->feature[id] >= 0) continue;
+                const float v = d->value[id];
+                if (!std::isfinite(v)) { finite = false; break; }
+                if (v == 0.0f) continue;
+                int e2 = 0;
+                std::frexp(v, &e2);                       // |v| in [2^(e2-1), 2^e2)
+                min_lsb = std::min(min_lsb, std::max(e2 - 24, -149));
+                max_e = std::max(max_e, e2);
+            }
+        if (finite) {
+            if (max_e == -(1 << 30)) { fx_ok = 1; fx_s = 0; }   // all leaves zero
+            else {
+                fx_s = -min_lsb;
+                int lg = 0;
+                while ((1LL << lg) < (long long)d->n_trees + 1) ++lg;
+                fx_ok = (max_e + fx_s + lg <= 61) ? 1 : 0;
+            }
         }
     }
     const int pad_leaf = (int)nodes.size();
@@ -548,6 +623,9 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
     m->dm.bdepth = bdepth;
+    m->dm.fx_ok = fx_ok;
+    m->dm.fx_scale = std::ldexp(1.0, fx_s);
+    m->dm.fx_inv = std::ldexp(1.0, -fx_s);
     *out = m;
     return ok();
 }
@@ -584,10 +662,22 @@ syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, sy
         if (!(h[i - 1] < h[i])) return fail(SYN_ERR_INVALID_ARG, "freqs not strictly ascending at %d", i);
     DeviceGuard g(device);
     if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
+    // clock-cut hint grid: grid[b] = #{i : f_i < f_0 + b * step}, b = 0..kGrid (any rounding is
+    // fine: the kernels finish every cut with exact comparisons against the table)
+    const float f0 = h[0], span = h[n_f - 1] - h[0];
+    const float step = span > 0.0f ? span / (float)kGrid : 1.0f;
+    std::vector<unsigned short> grid(kGrid + 1);
+    for (int b = 0; b <= kGrid; ++b) {
+        const float edge = f0 + (float)b * step;
+        grid[b] = (unsigned short)(std::lower_bound(h, h + n_f, edge) - h);
+    }
     float* d = nullptr;
-    cudaError_t e = cudaMalloc(&d, (size_t)n_f * sizeof(float));
+    const size_t gbytes = (size_t)(kGrid + 1) * sizeof(unsigned short);
+    const size_t goff = ((size_t)n_f * sizeof(float) + 255) / 256 * 256;
+    cudaError_t e = cudaMalloc(&d, goff + gbytes);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(clocks)");
-    if ((e = cudaMemcpy(d, h, (size_t)n_f * sizeof(float), cudaMemcpyHostToDevice)) != cudaSuccess) {
+    if ((e = cudaMemcpy(d, h, (size_t)n_f * sizeof(float), cudaMemcpyHostToDevice)) != cudaSuccess ||
+        (e = cudaMemcpy(reinterpret_cast<char*>(d) + goff, grid.data(), gbytes, cudaMemcpyHostToDevice)) != cudaSuccess) {
         cudaFree(d);
         return cuda_fail(e, "cudaMemcpy(clocks)");
     }
@@ -599,6 +689,9 @@ syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, sy
     c->device = device;
     c->n_f = n_f;
     c->d_freqs = d;
+    c->d_grid = reinterpret_cast<unsigned short*>(reinterpret_cast<char*>(d) + goff);
+    c->f0 = f0;
+    c->inv_step = 1.0f / step;
     *out = c;
     return ok();
 }

@@ -3,7 +3,7 @@
 OUT=gpurun_out/${1:-ab}
 mkdir -p $OUT
 for c in ${CFGS:-c2 c3 c5 c4 c1}; do
-  for algo in interval direct; do
+  for algo in ${ALGOS:-da ws direct}; do
     SYNERGY_ALGO=$algo timeout 600 python bench.py --config $c --steps ${STEPS:-20} --warmup 3 --no-cpu-baseline --no-e2e > $OUT/$c.$algo.json 2> $OUT/$c.$algo.err
     python -c "
 import json,sys

@@ -22,7 +22,10 @@ def _build():
 
 
 # Kernel variants the library can pick (read per call from the environment):
-#   default   warp-streaming clock-interval kernel (k_sweep_ws), 2 kernels per CTA, window 48
+#   default   order-free difference-array kernel (k_sweep_da), exact int64 leaf sums
+#   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
+#   da_nt256  k_sweep_da with 256 threads per kernel (idle lanes on small forests)
+#   ws        in-order warp-streaming kernel (k_sweep_ws), 2 kernels per CTA, window 64
 #   ws_tight  k_sweep_ws with window 32 (= warp width: refills wait on the oldest tree), 1 run
 #             value kept per tree (every later run takes the direct-walk fallback), 3 kernels/CTA
 #   ws_wide   k_sweep_ws with window 128, 1 kernel per CTA
@@ -31,7 +34,10 @@ def _build():
 #   iv_vcap1  k_sweep_iv keeping 1 run value per (kernel, tree)
 #   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
-VARIANTS = {"default": {}, "ws_tight": {"SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"}, "ws_wide": {"SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
+VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERGY_NT": "256"},
+            "ws": {"SYNERGY_ALGO": "ws"},
+            "ws_tight": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"},
+            "ws_wide": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
             "direct": {"SYNERGY_ALGO": "direct"}, "iv": {"SYNERGY_ALGO": "iv"},
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
@@ -101,6 +107,49 @@ def test_fuzz_bit_exact(case, variant):
         assert_bits_equal(got["S"], ref["S"], "S")
         assert_bits_equal(got["E"], ref["E"], "E")
         assert_choices(got["choice"], ref["choice"], ref["gap"])
+
+
+def _stump_models(values_S, values_E, F=3):
+    def spec(vals):
+        T = len(vals)
+        return W.ModelSpec(n_inputs=F + 1, forest_weight=1.0, tree_offset=np.arange(T + 1, dtype=np.int64),
+                           feature=np.full(T, -1, np.int32), left=np.full(T, -1, np.int32),
+                           right=np.full(T, -1, np.int32), value=np.asarray(vals, np.float32))
+    w = W.fuzz_workload(9, 4, 16, F=F)
+    w.speedup, w.energy = spec(values_S), spec(values_E)
+    return w
+
+
+def test_exact_sum_where_sequential_fp64_rounds():
+    """Leaves spanning 2^24 .. 2^-30 ulps: the int64 path (k_sweep_da) is exact like the oracle,
+    while a sequential fp64 sum of these leaves rounds (Q8)."""
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    big = float(np.float32(2.0 ** 24 + 2.0))
+    vals = [big, 0.008606708608567715, -big, 0.008446695283055305, big, 0.008703862316906452]
+    vals = [float(np.float32(v)) for v in vals]
+    import math
+    seq = 0.0
+    for v in vals:
+        seq += v
+    assert seq != math.fsum(vals)                             # the case really needs exactness
+    w = _stump_models(vals, [1.0, 2.0])
+    S, E = gpu_predict(w, default_idx=-1)
+    rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
+    assert syn.last_launch()["variant"] // 1000 == 3          # difference-array kernel ran
+    assert_bits_equal(S, rS, "raw S")
+    assert_bits_equal(E, rE, "raw E")
+
+
+def test_out_of_range_leaves_fall_back_to_ordered_kernel():
+    """Leaves spanning more than the int64 fixed-point range route to the ordered kernels; with
+    two leaves per evaluation the sequential fp64 sum is a single rounding = the exact sum."""
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = _stump_models([2.0 ** 60, 2.0 ** -60], [1.0, 0.5])
+    S, E = gpu_predict(w, default_idx=-1)
+    rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
+    assert syn.last_launch()["variant"] // 1000 != 3
+    assert_bits_equal(S, rS, "raw S")
+    assert_bits_equal(E, rE, "raw E")
 
 
 def test_empty_batch_is_noop():
