@@ -195,6 +195,22 @@ def oracle_single_core(cfg, n_k_cap, budget_s=10.0):
     return evals / el, evals, el
 
 
+def run_walk_work(cfg, row0, n_rows, cap=1000):
+    """Run-walk work of the launched rows, counted by the oracle on the first min(n_rows, cap)
+    rows (exact when n_rows <= cap): runs of clocks sharing a leaf and their 2-level block fetches."""
+    import oracle
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    n = min(n_rows, cap)
+    if n == 0:
+        return None
+    w = W.make_config(cfg, row0=row0, n=n)
+    r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
+    trees = w.speedup.n_trees + w.energy.n_trees
+    return {"run_blocks_per_kernel": r["run_blocks"] / n, "runs_per_kernel_tree": r["runs"] / (n * max(trees, 1)),
+            "sample": f"rows [{row0}, {row0 + n}) of {cfg}" + (" (all launched rows)" if n == n_rows else
+                                                             f" scaled to {n_rows} rows")}
+
+
 def run_reference(args, rank, world):
     """Reference arm: the CPU oracle (as it stands, single-threaded per process) on the box's host
     cores, one process per core over contiguous kernel ranges of a bounded sample per step."""
@@ -375,21 +391,43 @@ def main():
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     dec = decisions_per_eval(sp_spec) + decisions_per_eval(en_spec)
     kern_avg_s = statistics.mean(kern_ms) / 1e3
-    achieved = evals_step * dec / kern_avg_s / 1e9                  # G node-decisions / s
-    # on-chip ceiling: one warp-level node decision needs >= 2 L1/shared
-    # wavefronts (node load + feature load), 1 wavefront/clk/SM -> 16 lane-decisions/clk/SM
-    peak = sms * sm_max * 1e6 * 32 / 2 / 1e9
+    variant = syn.last_launch()["variant"]
+    algo = {0: "k_sweep", 1: "k_sweep_iv", 2: "k_sweep_ws", 3: "k_sweep_da"}[variant // 1000 if variant >= 1000 else 0]
     hbm_bytes = evals_step // n_f * (W.N_STATIC * 4 + n_t * 4) + n_f * 4 + \
         sp.info()["device_bytes"] + en.info()["device_bytes"]
     hbm_ach = hbm_bytes / kern_avg_s / 1e9
-    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
-                "frac": achieved / peak, "traffic": ncu_traffic(cfg),
-                "kernel": "k_sweep", "kernel_ms": statistics.mean(kern_ms),
-                "kernel_share_of_step": sum(kern_ms) / total_ms,
-                "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
-                "hbm": {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                        "frac": hbm_ach / peaks["hbm_gbs"], "algorithmic_bytes": hbm_bytes,
-                        "peak_source": peak_src}}
+    hbm = {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": hbm_ach / peaks["hbm_gbs"],
+           "algorithmic_bytes": hbm_bytes, "peak_source": peak_src}
+    work = None
+    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws"):
+        work = run_walk_work(cfg, row0, n_local)
+    if work is not None:
+        # on-chip L1 roofline: each run walk fetches max(1, ceil(depth/2)) 32-byte
+        # 2-level blocks; counted by the oracle from the inputs (runs of clocks sharing a leaf)
+        blocks = work["run_blocks_per_kernel"] * (evals_step // n_f)
+        achieved = 32.0 * blocks / kern_avg_s / 1e9
+        peak = 128.0 * sms * sm_max * 1e6 / 1e9
+        roofline = {"bound": "l1", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                    "traffic": ncu_traffic(cfg), "kernel": algo, "kernel_ms": statistics.mean(kern_ms),
+                    "kernel_share_of_step": sum(kern_ms) / total_ms,
+                    "algorithmic_bytes_per_launch": 32.0 * blocks,
+                    "work": {"unit": "32-byte 2-level block fetches of the run walks", "per_launch": blocks,
+                             "runs_per_kernel_tree": work["runs_per_kernel_tree"], "counted_on": work["sample"]},
+                    "peak_note": f"L1/TEX load path 128 B/clk/SM x {sms} SMs x {sm_max:.0f} MHz (derived; "
+                                 "not in MEASURED_PEAKS.json)",
+                    "l1_wavefront_view": {"achieved_per_s": 2.0 * blocks / kern_avg_s,
+                                          "peak_per_s": sms * sm_max * 1e6,
+                                          "note": "scattered walks: each 16-byte load is one wavefront, 2 per block"},
+                    "decisions_per_s_vs_direct": evals_step * dec / kern_avg_s,
+                    "hbm": hbm}
+    else:
+        achieved = evals_step * dec / kern_avg_s / 1e9                  # G node-decisions / s
+        peak = sms * sm_max * 1e6 * 32 / 2 / 1e9
+        roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
+                    "frac": achieved / peak, "traffic": ncu_traffic(cfg), "kernel": algo,
+                    "kernel_ms": statistics.mean(kern_ms), "kernel_share_of_step": sum(kern_ms) / total_ms,
+                    "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
+                    "hbm": hbm}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

@@ -64,6 +64,16 @@ int oracle_sweep(const oracle_model *speedup, const oracle_model *energy,
                  const int32_t *kind, const float *x, int32_t n_t,
                  int32_t *choice, float *S, float *E, double *gap, int64_t *visits);
 
+/* oracle_sweep plus work counters of the run-walk algorithm (DESIGN.md §6 roofline): runs =
+ * maximal clock runs sharing a leaf per (kernel, tree), run_decisions = sum of their leaf depths,
+ * run_blocks = sum of max(1, ceil(depth/2)).  Counters are added to (not reset). */
+int oracle_sweep_stats(const oracle_model *speedup, const oracle_model *energy,
+                       const float *features, int64_t n_k, int32_t n_features,
+                       const float *freqs, int32_t n_f, int32_t default_idx,
+                       const int32_t *kind, const float *x, int32_t n_t,
+                       int32_t *choice, int64_t *visits, int64_t *runs, int64_t *run_decisions,
+                       int64_t *run_blocks);
+
 #ifdef __cplusplus
 }
 #endif

@@ -256,42 +256,52 @@ cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaS
     return launch_ws_t<8>(a, c, grid, st);
 }
 
-// Difference-array kernel: one CTA per kernel, exact int64 leaf sums (needs fx_ok forests).
+// Difference-array kernel: KPC kernels per CTA, exact int64 leaf sums (needs fx_ok forests).
+// KPC grows when a kernel has fewer trees than the CTA has threads, so lanes keep walking and
+// the per-CTA staging / finish is amortised.
+size_t da_smem(int nt, int kpc, int n_f, int xs) {
+    return (size_t)kpc * 2 * (n_f + 1) * 8 + (size_t)nt * kpc * 2 * 8 + (size_t)kpc * n_f * 24 +
+           (size_t)n_f * 4 + (size_t)kpc * xs * 4 + (size_t)(kGrid + 2) * 2 + 16;
+}
+
 bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c) {
     if (n_f > 2048) return false;
     if ((sp->n_trees && !sp->dm.fx_ok) || (en->n_trees && !en->dm.fx_ok)) return false;
     const int tt = sp->n_trees + en->n_trees;
-    int nt = env_int("SYNERGY_NT", tt > 256 ? 256 : 128);
+    int nt = env_int("SYNERGY_NT", 128);
     nt = nt >= 256 ? 256 : (nt >= 128 ? 128 : 64);
+    int kpc = tt >= nt ? 1 : (3 * nt + 2 * tt - 1) / (2 * tt);      // ~1.5 tasks per thread
+    kpc = env_int("SYNERGY_KPC", kpc);
+    kpc = (int)std::max<long long>(1, std::min<long long>(std::min(kpc, 16), std::max<long long>(n_k, 1)));
     c.algo = 3;
     c.slots = c.tilp = 0;
-    c.tile_k = 1;
+    c.tile_k = kpc;
     c.nt = nt;
     c.xs = (F + 2) | 1;
     c.tc = c.words = c.vcap = c.vs = c.region = 0;
     c.win = c.slot_bytes = c.head_bytes = 0;
-    c.smem = (size_t)2 * (n_f + 1) * 8 + (size_t)n_f * 24 + (size_t)n_f * 4 + (size_t)c.xs * 4 +
-             (size_t)((kGrid + 2) & ~1) * 2 + 16;
-    (void)n_k;
-    return c.smem <= 220 * 1024;
+    c.smem = da_smem(nt, kpc, n_f, c.xs);
+    while (c.smem > 200 * 1024 && c.tile_k > 1) c.smem = da_smem(nt, --c.tile_k, n_f, c.xs);
+    return c.smem <= 200 * 1024;
 }
 
-template <int NT>
+template <int NT, bool PAIR>
 cudaError_t launch_da_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
     static size_t smem_set = 48 * 1024;
     if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT, PAIR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
         if (e != cudaSuccess) return e;
         smem_set = c.smem;
     }
-    k_sweep_da<NT><<<(unsigned)grid, NT, c.smem, st>>>(a);
+    k_sweep_da<NT, PAIR><<<(unsigned)grid, NT, c.smem, st>>>(a);
     return cudaGetLastError();
 }
 
 cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    if (c.nt == 256) return launch_da_t<256>(a, c, grid, st);
-    if (c.nt == 128) return launch_da_t<128>(a, c, grid, st);
-    return launch_da_t<64>(a, c, grid, st);
+    const bool pair = env_int("SYNERGY_PAIR", 0) != 0;
+    if (c.nt == 256) return pair ? launch_da_t<256, true>(a, c, grid, st) : launch_da_t<256, false>(a, c, grid, st);
+    if (c.nt == 128) return pair ? launch_da_t<128, true>(a, c, grid, st) : launch_da_t<128, false>(a, c, grid, st);
+    return pair ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
 }
 
 template <int S, int T>

@@ -1,0 +1,60 @@
+"""Pins for the oracle's run-walk work counters (oracle.c: oracle_sweep_stats), the numerator of
+the k_sweep_da roofline.  Checked against an independent formulation: a depth-first
+walk of each tree over the clock-index interval that splits at clock thresholds (each leaf reached
+owns one run of consecutive clocks), written here from the tree definition."""
+import numpy as np
+
+from paper_conf_sc_fandccfc23_b200 import workloads as W
+
+
+def interval_runs(spec, t, x_static, freqs):
+    """(runs, sum of leaf depths, sum of max(1, ceil(depth/2))) for one (kernel, tree)."""
+    base = spec.tree_offset[t]
+    F = len(x_static)
+    runs = dec = blk = 0
+    stack = [(0, 0, len(freqs), 0)]
+    while stack:
+        n, lo, hi, d = stack.pop()
+        f = spec.feature[base + n]
+        if f < 0:
+            runs += 1
+            dec += d
+            blk += max(1, (d + 1) // 2)
+            continue
+        thr = spec.value[base + n]
+        L, R = spec.left[base + n], spec.right[base + n]
+        if f < F:
+            stack.append((L if x_static[f] <= thr else R, lo, hi, d + 1))
+            continue
+        s = int(np.searchsorted(freqs, thr, side="right"))     # #clocks <= thr
+        if s < hi and max(s, lo) < hi:
+            stack.append((R, max(s, lo), hi, d + 1))
+        if s > lo:
+            stack.append((L, lo, min(s, hi), d + 1))
+    return runs, dec, blk
+
+
+def _check(w):
+    import oracle
+    r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
+    runs = dec = blk = 0
+    for k in range(w.n_kernels):
+        for m in (w.speedup, w.energy):
+            if m.forest_weight == 0.0:
+                continue
+            for t in range(m.n_trees):
+                a, b, c = interval_runs(m, t, w.features[k], w.freqs)
+                runs += a
+                dec += b
+                blk += c
+    assert (r["runs"], r["run_decisions"], r["run_blocks"]) == (runs, dec, blk)
+    np.testing.assert_array_equal(r["choice"], oracle.sweep_workload(w)["choice"])
+
+
+def test_workcount_c1():
+    _check(W.make_config("c1"))
+
+
+def test_workcount_fuzz_unbalanced_exact_thresholds():
+    for seed in range(4):
+        _check(W.fuzz_workload(50 + seed, 5, 33, F=4, n_trees=4, max_depth=7, exact_thresholds=True))
