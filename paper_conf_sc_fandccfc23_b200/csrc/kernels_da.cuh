@@ -18,9 +18,10 @@
 // reaches, exactly.  Then forest = (double)acc * 2^-s / T, linear member, default-clock
 // normalisation and per-target argmin (finish_tile) as everywhere else.
 //
-// Block loads are lane-paired: lanes 2i and 2i+1 fetch the two 16-byte halves of the SAME 32-byte
-// block in one instruction (one L1 sector for two lanes, the L1 wavefront rate being the bound of
-// this kernel), then trade the one grandchild word each needs with a shuffle.
+// The kernel is bound by the L1 wavefront rate of the scattered block loads.  Every restart walk
+// of a task re-traverses the top of the same tree, so at task start each thread stages the root
+// block and its four grandchild blocks (the top two block levels, 160 B) in shared memory and the
+// walks read levels 0-1 from there (TOPC; about a quarter fewer global block loads per task).
 #pragma once
 #include "kernels_ws.cuh"
 
@@ -30,69 +31,16 @@ __device__ __forceinline__ void atomic_add_s64(long long* p, long long v) {
     atomicAdd(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);   // two's complement
 }
 
-// Clock cut with the hint grid read through L1 (built once per clock table, syn_clocks).
-__device__ __forceinline__ int clock_cut_g(unsigned fr_a, const unsigned short* __restrict__ grid,
-                                           float f0, float inv_step, float thr, int lo, int hi) {
-    int b = __float2int_rz((thr - f0) * inv_step);
-    b = min(max(b, 0), kGrid);
-    int s = min(max((int)__ldg(grid + b), lo + 1), hi - 1);
-    while (s > lo + 1 && !(lds_f(fr_a + 4u * (s - 1)) <= thr)) --s;
-    while (s < hi - 1 && lds_f(fr_a + 4u * s) <= thr) ++s;
-    return s;
+__device__ __forceinline__ void sts_blk(unsigned a, uint4 v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w));
+}
+__device__ __forceinline__ uint4 lds_blk(unsigned a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
 }
 
-// One lane-paired 2-level block step, executed by all 32 lanes (warp-synchronous).  Lane state:
-// bk = block index in its own model's array, isE = model, done = no walk / walk finished.
-__device__ __forceinline__ void pair_block_step(const uint4* __restrict__ bS, const uint4* __restrict__ bE,
-                                                int& bk, bool isE, bool& done, float& leaf, float& tmin,
-                                                float f, unsigned xrow_a, int F, bool odd) {
-    const int info = done ? -1 : ((bk << 1) | (isE ? 1 : 0));
-    const int pinfo = __shfl_xor_sync(0xffffffffu, info, 1);
-    const int xinfo = odd ? pinfo : info;            // the even lane's block
-    const int yinfo = odd ? info : pinfo;            // the odd lane's block
-    uint4 r1 = make_uint4(0u, 0u, 0u, 0u), r2 = make_uint4(0u, 0u, 0u, 0u);
-    if (xinfo >= 0) r1 = ldg_blk(((xinfo & 1) ? bE : bS) + 2 * (size_t)(xinfo >> 1) + (odd ? 1 : 0));
-    if (yinfo >= 0) r2 = ldg_blk(((yinfo & 1) ? bE : bS) + 2 * (size_t)(yinfo >> 1) + (odd ? 0 : 1));
-    const uint4 A = odd ? r2 : r1;                   // own block, words 0..3
-    const uint4 Bp = odd ? r1 : r2;                  // partner's block, words 4..7
-    int slot = 0;
-    bool need = false;
-    if (!done) {
-        const unsigned codes = A.w;
-        const int cn = (int)(codes & 0xffu);
-        const float tn = __uint_as_float(A.x);
-        if (cn > F) {                                // one-leaf tree
-            leaf = tn;
-            done = true;
-        } else {
-            const float xn = (cn == F) ? f : lds_f(xrow_a + 4u * (unsigned)cn);
-            const bool r0 = !(xn <= tn);
-            if (cn == F && !r0) tmin = fminf(tmin, tn);
-            const float tc = __uint_as_float(r0 ? A.z : A.y);
-            const int cc = (int)((codes >> (r0 ? 16 : 8)) & 0xffu);
-            if (cc > F) {                            // child leaf (odd depth)
-                leaf = tc;
-                done = true;
-            } else {
-                const float xc = (cc == F) ? f : lds_f(xrow_a + 4u * (unsigned)cc);
-                const bool r1b = !(xc <= tc);
-                if (cc == F && !r1b) tmin = fminf(tmin, tc);
-                slot = (r0 ? 2 : 0) + (r1b ? 1 : 0);
-                need = true;
-                if ((codes >> (24 + slot)) & 1u) done = true;   // grandchild is a leaf
-            }
-        }
-    }
-    const int pslot = __shfl_xor_sync(0xffffffffu, slot, 1);
-    const unsigned give = pslot == 0 ? Bp.x : pslot == 1 ? Bp.y : pslot == 2 ? Bp.z : Bp.w;
-    const unsigned g = __shfl_xor_sync(0xffffffffu, give, 1);
-    if (need) {
-        if (done) leaf = __uint_as_float(g);
-        else bk = (int)g;
-    }
-}
-
-template <int NT, bool PAIR>
+template <int NT, bool TOPC>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constant__ SweepArgs a) {
     extern __shared__ __align__(16) unsigned char smem[];
     const int n_f = a.n_f, F = a.F, XS = a.xs, KPC = a.tile_k;
@@ -108,6 +56,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
     float* xk = fr + n_f;                                                   // [KPC][XS]
     unsigned short* grid = reinterpret_cast<unsigned short*>(xk + KPC * XS);   // [kGrid + 2]
     int* counter = reinterpret_cast<int*>(grid + kGrid + 2);
+    // per-thread cache of its task's top two block levels: root + 4 grandchild blocks (5 x 32 B)
+    uint4* topc = reinterpret_cast<uint4*>(smem + a.head_bytes);
 
     const float* gfeat = a.features + k0 * F;
     for (int e = threadIdx.x; e < nk * F; e += NT) {
@@ -127,9 +77,9 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
     __syncthreads();
 
     const int lane = threadIdx.x & 31;
-    const bool odd = lane & 1;
     const unsigned lm_lt = lanemask_lt();
     const unsigned xk_a = su32(xk), fr_a = su32(fr), grid_a = su32(grid);
+    const unsigned topc_a = su32(topc) + (unsigned)threadIdx.x * 160u;
     const float f0 = a.f0, inv_step = a.inv_step;
     const float f_last = fr[n_f - 1];
     const int TS = a.ms.forest_weight != 0.0 ? a.ms.n_trees : 0;
@@ -169,6 +119,23 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
                     scale = m.fx_scale;
                     root = __ldg(m.broot + (isE ? jj - TS : jj));
                     xrow_a = xk_a + 4u * (unsigned)(kl * XS);
+                    if (TOPC) {                               // stage the top two block levels
+                        const uint4* bl = isE ? bE : bS;
+                        const uint4 A0 = ldg_blk(bl + 2 * (size_t)root), B0 = ldg_blk(bl + 2 * (size_t)root + 1);
+                        sts_blk(topc_a, A0);
+                        sts_blk(topc_a + 16u, B0);
+                        const unsigned cw = A0.w;
+                        const unsigned gs[4] = {B0.x, B0.y, B0.z, B0.w};
+#pragma unroll
+                        for (int s2 = 0; s2 < 4; ++s2) {
+                            const bool inner = (int)(cw & 0xffu) <= F && (int)((cw >> (8 + 8 * (s2 >> 1))) & 0xffu) <= F &&
+                                               !((cw >> (24 + s2)) & 1u);
+                            if (inner) {
+                                sts_blk(topc_a + 32u * (1 + s2), ldg_blk(bl + 2 * (size_t)gs[s2]));
+                                sts_blk(topc_a + 32u * (1 + s2) + 16u, ldg_blk(bl + 2 * (size_t)gs[s2] + 1));
+                            }
+                        }
+                    }
                     lo = 0;
                     f_lo = lds_f(fr_a);
                     tmin = CUDART_INF_F;
@@ -182,11 +149,18 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
         float leaf = 0.0f;
         int bk = root;
         bool done = task < 0;
-        if (PAIR) {
-            for (int d = 0; d < BD; ++d)
-                pair_block_step(bS, bE, bk, isE, done, leaf, tmin, f_lo, xrow_a, F, odd);
+        const uint4* __restrict__ own = isE ? bE : bS;
+        if (TOPC) {                                   // levels 0-1 from the shared cache
+            int gs = 0;
+            if (!done) block_decide(lds_blk(topc_a), lds_blk(topc_a + 16u), bk, gs, done, leaf, tmin, f_lo, xrow_a, F);
+            if (BD > 1 && !done) {
+                const unsigned ca = topc_a + 32u * (1 + gs);
+                block_decide(lds_blk(ca), lds_blk(ca + 16u), bk, gs, done, leaf, tmin, f_lo, xrow_a, F);
+            }
+#pragma unroll 2
+            for (int d = 2; d < BD; ++d)
+                if (!done) block_step(own, bk, done, leaf, tmin, f_lo, xrow_a, F);
         } else {
-            const uint4* __restrict__ own = isE ? bE : bS;
 #pragma unroll 2
             for (int d = 0; d < BD; ++d)
                 if (!done) block_step(own, bk, done, leaf, tmin, f_lo, xrow_a, F);

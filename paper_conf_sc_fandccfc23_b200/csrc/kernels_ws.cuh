@@ -71,13 +71,12 @@ __device__ __forceinline__ uint4 ldg_blk(const uint4* p) {
     return r;
 }
 
-// One 2-level block step (internal.h layout) for clock value f: decides at the block's node and
-// at the chosen child, records the smallest left-turn clock threshold in tmin, and either moves
-// b to the chosen grandchild block or sets leaf + done.
-__device__ __forceinline__ void block_step(const uint4* __restrict__ blocks, int& b, bool& done,
-                                           float& leaf, float& tmin, float f, unsigned xrow_a, int F) {
-    const uint4 A = ldg_blk(blocks + 2 * (size_t)b);
-    const uint4 B = ldg_blk(blocks + 2 * (size_t)b + 1);
+// Decide one 2-level block (internal.h layout) already in registers (A = words 0..3, B = 4..7)
+// for clock value f: decides at the block's node and at the chosen child, records the smallest
+// left-turn clock threshold in tmin, and either moves b to the chosen grandchild block (gslot =
+// its slot 0..3) or sets leaf + done.
+__device__ __forceinline__ void block_decide(const uint4 A, const uint4 B, int& b, int& gslot, bool& done,
+                                             float& leaf, float& tmin, float f, unsigned xrow_a, int F) {
     const unsigned codes = A.w;
     const int cn = (int)(codes & 0xffu);
     const float tn = __uint_as_float(A.x);
@@ -106,7 +105,17 @@ __device__ __forceinline__ void block_step(const uint4* __restrict__ blocks, int
         done = true;
     } else {
         b = (int)g;
+        gslot = slot;
     }
+}
+
+// One 2-level block step loading the block from global memory (read-only path).
+__device__ __forceinline__ void block_step(const uint4* __restrict__ blocks, int& b, bool& done,
+                                           float& leaf, float& tmin, float f, unsigned xrow_a, int F) {
+    const uint4 A = ldg_blk(blocks + 2 * (size_t)b);
+    const uint4 B = ldg_blk(blocks + 2 * (size_t)b + 1);
+    int gs = 0;
+    block_decide(A, B, b, gs, done, leaf, tmin, f, xrow_a, F);
 }
 
 __device__ __forceinline__ unsigned lanemask_lt() {

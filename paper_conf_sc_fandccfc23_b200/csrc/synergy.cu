@@ -259,9 +259,14 @@ cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaS
 // Difference-array kernel: KPC kernels per CTA, exact int64 leaf sums (needs fx_ok forests).
 // KPC grows when a kernel has fewer trees than the CTA has threads, so lanes keep walking and
 // the per-CTA staging / finish is amortised.
+size_t da_head(int nt, int kpc, int n_f, int xs) {
+    const size_t h = (size_t)kpc * 2 * (n_f + 1) * 8 + (size_t)nt * kpc * 2 * 8 + (size_t)kpc * n_f * 24 +
+                     (size_t)n_f * 4 + (size_t)kpc * xs * 4 + (size_t)(kGrid + 2) * 2 + 16;
+    return (h + 15) & ~(size_t)15;
+}
+
 size_t da_smem(int nt, int kpc, int n_f, int xs) {
-    return (size_t)kpc * 2 * (n_f + 1) * 8 + (size_t)nt * kpc * 2 * 8 + (size_t)kpc * n_f * 24 +
-           (size_t)n_f * 4 + (size_t)kpc * xs * 4 + (size_t)(kGrid + 2) * 2 + 16;
+    return da_head(nt, kpc, n_f, xs) + (size_t)nt * 160;   // + per-thread top-block cache
 }
 
 bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c) {
@@ -271,6 +276,7 @@ bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f,
     int nt = env_int("SYNERGY_NT", 128);
     nt = nt >= 256 ? 256 : (nt >= 128 ? 128 : 64);
     int kpc = tt >= nt ? 1 : (3 * nt + 2 * tt - 1) / (2 * tt);      // ~1.5 tasks per thread
+    kpc = (int)std::min<long long>(kpc, std::max<long long>(1, n_k / (2LL * sm_count(0))));   // fill the SMs
     kpc = env_int("SYNERGY_KPC", kpc);
     kpc = (int)std::max<long long>(1, std::min<long long>(std::min(kpc, 16), std::max<long long>(n_k, 1)));
     c.algo = 3;
@@ -282,26 +288,27 @@ bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f,
     c.win = c.slot_bytes = c.head_bytes = 0;
     c.smem = da_smem(nt, kpc, n_f, c.xs);
     while (c.smem > 200 * 1024 && c.tile_k > 1) c.smem = da_smem(nt, --c.tile_k, n_f, c.xs);
+    c.head_bytes = (int)da_head(nt, c.tile_k, n_f, c.xs);
     return c.smem <= 200 * 1024;
 }
 
-template <int NT, bool PAIR>
+template <int NT, bool TOPC>
 cudaError_t launch_da_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
     static size_t smem_set = 48 * 1024;
     if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT, PAIR>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
+        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT, TOPC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
         if (e != cudaSuccess) return e;
         smem_set = c.smem;
     }
-    k_sweep_da<NT, PAIR><<<(unsigned)grid, NT, c.smem, st>>>(a);
+    k_sweep_da<NT, TOPC><<<(unsigned)grid, NT, c.smem, st>>>(a);
     return cudaGetLastError();
 }
 
 cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    const bool pair = env_int("SYNERGY_PAIR", 0) != 0;
-    if (c.nt == 256) return pair ? launch_da_t<256, true>(a, c, grid, st) : launch_da_t<256, false>(a, c, grid, st);
-    if (c.nt == 128) return pair ? launch_da_t<128, true>(a, c, grid, st) : launch_da_t<128, false>(a, c, grid, st);
-    return pair ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
+    const bool topc = env_int("SYNERGY_TOPC", 1) != 0;
+    if (c.nt == 256) return topc ? launch_da_t<256, true>(a, c, grid, st) : launch_da_t<256, false>(a, c, grid, st);
+    if (c.nt == 128) return topc ? launch_da_t<128, true>(a, c, grid, st) : launch_da_t<128, false>(a, c, grid, st);
+    return topc ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
 }
 
 template <int S, int T>

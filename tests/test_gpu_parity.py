@@ -26,7 +26,7 @@ def _build():
 #   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
 #   da_nt256  k_sweep_da with 256 threads per CTA
 #   da_kpc5   k_sweep_da with 5 kernels per CTA (tasks of several kernels per warp, ragged tile)
-#   da_pair   k_sweep_da with lane-paired block loads, 3 kernels per CTA
+#   da_notopc k_sweep_da without the shared top-block cache, 3 kernels per CTA
 #   ws        in-order warp-streaming kernel (k_sweep_ws), 2 kernels per CTA, window 64
 #   ws_tight  k_sweep_ws with window 32 (= warp width: refills wait on the oldest tree), 1 run
 #             value kept per tree (every later run takes the direct-walk fallback), 3 kernels/CTA
@@ -37,7 +37,7 @@ def _build():
 #   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
 VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERGY_NT": "256"},
-            "da_kpc5": {"SYNERGY_KPC": "5"}, "da_pair": {"SYNERGY_PAIR": "1", "SYNERGY_KPC": "3"},
+            "da_kpc5": {"SYNERGY_KPC": "5"}, "da_notopc": {"SYNERGY_TOPC": "0", "SYNERGY_KPC": "3"},
             "ws": {"SYNERGY_ALGO": "ws"},
             "ws_tight": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"},
             "ws_wide": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
@@ -45,7 +45,7 @@ VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERG
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_PAIR")
+KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC")
 
 
 @pytest.fixture(params=list(VARIANTS))
