@@ -12,7 +12,7 @@
  *   of kernels with a speedup model and an energy model, normalises both to the default
  *   clock, and returns one clock index per kernel per target.  The readings of points the
  *   paper leaves open are DESIGN.md Q1-Q23 (exhaustive lowest-index argmin, potential-saving
- *   ES/PL, x <= threshold goes left, fp64 accumulation, ...).
+ *   ES/PL, x <= threshold goes left, exact leaf sums, ...).
  *
  * Conventions for every call:
  *   - All calls return syn_status; no C++ exception crosses the ABI.  On a non-OK status the
@@ -78,8 +78,9 @@ typedef void *syn_stream;   /* cudaStream_t */
  * in MHz; inputs 0..n_inputs-2 are the static features.  Output (Q7/Q8):
  *   m(x) = 0;  m += linear_weight * (lin_b + sum_j lin_w[j] x[j])   if linear_weight != 0
  *              m += forest_weight * mean_t leaf_t(x)                if forest_weight != 0
- * accumulated in fp64 (fp64 fma over j in order for the linear member, fp64 sum of the fp32
- * leaves in tree order, then / n_trees); a weight of exactly 1 skips its multiplication. */
+ * in fp64: fp64 fma over j in order for the linear member; for the forest the exact sum of the
+ * fp32 leaves rounded once to fp64 (order-free, Q8), then / n_trees; a weight of
+ * exactly 1 skips its multiplication. */
 typedef struct {
     int32_t n_inputs;            /* F + 1, 1 .. SYNERGY_MAX_INPUTS                        */
     double linear_weight;        /* 0 => no linear member                                 */
@@ -150,6 +151,20 @@ syn_status synergy_sweep(const syn_model *speedup, const syn_model *energy,
                          const syn_clocks *clocks, int32_t default_idx,
                          const syn_target *h_targets, int32_t n_targets, int32_t *d_choice,
                          float *d_speedup, float *d_energy, syn_stream stream);
+
+/* Four-model variant (single-target models F_t, F_e, F_edp, F_ed2p; Table 2
+ * "Best" pairs MIN_EDP with RandomForest, MIN_ED2P with Linear).  models[0] speedup, [1] energy,
+ * [2] direct EDP model, [3] direct ED2P model; [2] and [3] may be NULL (that target's key is then
+ * derived as E/S resp. E/S^2, as in synergy_sweep).  Each model is normalised by its own default-
+ * clock prediction; MIN_EDP / MIN_ED2P minimise the direct model's normalised prediction (a clock
+ * also needs that prediction finite and > 0).  d_pred (nullable): [4][n_kernels][n_freqs]
+ * normalised predictions (rows of absent models untouched).  Runs on the exact fixed-point kernel
+ * only: SYN_ERR_UNSUPPORTED when a forest's leaves exceed its int64 range (Q8).
+ * Other errors as synergy_sweep. */
+syn_status synergy_sweep4(const syn_model *const *models, const float *d_features, int64_t n_kernels,
+                          int32_t n_features, const syn_clocks *clocks, int32_t default_idx,
+                          const syn_target *h_targets, int32_t n_targets, int32_t *d_choice,
+                          float *d_pred, syn_stream stream);
 
 /* End-to-end host-buffer path: copies h_features host->device into the workspace, runs
  * synergy_sweep, copies the choices device->host into h_choice, all enqueued on `stream`

@@ -56,6 +56,9 @@ def _load():
         lib.oracle_select.restype = C.c_int
         lib.oracle_select.argtypes = [P, P, C.c_int64, C.c_int32, C.c_int32, P, P, C.c_int32,
                                       P, P]
+        lib.oracle_sweep4.restype = C.c_int
+        lib.oracle_sweep4.argtypes = [P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32, P, P,
+                                      C.c_int32, P, P]
         lib.oracle_sweep_stats.restype = C.c_int
         lib.oracle_sweep_stats.argtypes = [P, P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32,
                                            P, P, C.c_int32, P, P, P, P, P]
@@ -191,6 +194,24 @@ def sweep_stats(speedup, energy, features, freqs, default_idx, targets):
         raise OracleError("oracle_sweep_stats: invalid arguments")
     return {"choice": ch, "visits": int(c[0]), "runs": int(c[1]), "run_decisions": int(c[2]),
             "run_blocks": int(c[3])}
+
+
+def sweep4(models, features, freqs, default_idx, targets, want_pred=False):
+    """Four-model variant: models = [speedup, energy, edp|None, ed2p|None]."""
+    lib = _load()
+    keeps = [None if m is None else _Keep(m) for m in models]
+    arr = (C.c_void_p * 4)(*[None if k is None else C.cast(C.pointer(k.s), C.c_void_p) for k in keeps])
+    features = np.ascontiguousarray(features, dtype=np.float32)
+    freqs = np.ascontiguousarray(freqs, dtype=np.float32)
+    n_k, F = features.shape
+    kinds, xs = _targets(targets)
+    ch = np.empty((n_k, len(kinds)), np.int32)
+    P = np.empty((4, n_k, freqs.shape[0]), np.float32) if want_pred else None
+    rc = lib.oracle_sweep4(arr, _ptr(features), n_k, F, _ptr(freqs), freqs.shape[0], int(default_idx),
+                           _ptr(kinds), _ptr(xs), len(kinds), _ptr(ch), _ptr(P))
+    if rc != 0:
+        raise OracleError("oracle_sweep4: invalid arguments")
+    return {"choice": ch, "P": P} if want_pred else {"choice": ch}
 
 
 def sweep_workload(w, **kw):

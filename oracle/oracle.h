@@ -74,6 +74,13 @@ int oracle_sweep_stats(const oracle_model *speedup, const oracle_model *energy,
                        int32_t *choice, int64_t *visits, int64_t *runs, int64_t *run_decisions,
                        int64_t *run_blocks);
 
+/* Four-model variant: models[0] speedup, [1] energy, [2] EDP, [3] ED2P
+ * ([2]/[3] nullable = derived).  MIN_EDP / MIN_ED2P use the direct model's normalised
+ * prediction.  P (nullable) receives [4][n_k][n_f] normalised predictions. */
+int oracle_sweep4(const oracle_model *const *models, const float *features, int64_t n_k,
+                  int32_t n_features, const float *freqs, int32_t n_f, int32_t default_idx,
+                  const int32_t *kind, const float *x, int32_t n_t, int32_t *choice, float *P);
+
 #ifdef __cplusplus
 }
 #endif

@@ -51,6 +51,8 @@ enum Mode : int { kModePredict = 0, kModeSweep = 1 };
 
 struct SweepArgs {
     DevModel ms, me;         // speedup, energy
+    DevModel mx[2];          // four-model variant: direct EDP, ED2P models (k_sweep_da only)
+    int has_x[2];            // which of mx are present
     const float* features;   // [n_k][F]
     long long n_k;
     int F;                   // static features; clock is input F
@@ -63,6 +65,7 @@ struct SweepArgs {
     int* choice;             // [n_k][n_t] (sweep)
     float* S_out;            // [n_k][n_f] or null
     float* E_out;
+    float* X_out[2];         // direct EDP / ED2P normalised predictions, [n_k][n_f] or null
     int mode;
     int tile_k;              // kernels per CTA
     int xs;                  // x-vector stride in smem (floats)
@@ -79,6 +82,7 @@ struct SweepArgs {
     // clock-cut grid built once per clock table (syn_clocks)
     const unsigned short* grid;   // [kGrid + 1]
     float f0, inv_step;
+    int nsub;                // k_sweep_da: clock sub-ranges per (kernel, tree) task (small batches)
 };
 
 struct SelectArgs {

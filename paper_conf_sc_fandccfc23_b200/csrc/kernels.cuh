@@ -107,7 +107,8 @@ __device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
 
 // One warp selects all targets of one kernel from its n_f normalised predictions
 // (S, E in shared or global memory).  Writes out[0..n_t).
-__device__ __forceinline__ void select_row_warp(const float* S, const float* E, int n_f, int def,
+__device__ __forceinline__ void select_row_warp(const float* S, const float* E, const float* P2,
+                                                const float* P3, int n_f, int def,
                                                 int n_t, const int* kind, const float* xs,
                                                 int* out, int lane) {
     const float sd = S[def], ed = E[def];
@@ -141,8 +142,14 @@ __device__ __forceinline__ void select_row_warp(const float* S, const float* E, 
             switch (kd) {
                 case 0: key = -s; break;                                   // MAX_PERF
                 case 1: key = e; break;                                    // MIN_ENERGY
-                case 2: key = __ddiv_rn(e, s); break;                      // MIN_EDP  e*t
-                case 3: key = __ddiv_rn(__ddiv_rn(e, s), s); break;        // MIN_ED2P e*t^2
+                case 2:                                                    // MIN_EDP  e*t
+                    if (P2) { const float p = P2[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
+                    else key = __ddiv_rn(e, s);
+                    break;
+                case 3:                                                    // MIN_ED2P e*t^2
+                    if (P3) { const float p = P3[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
+                    else key = __ddiv_rn(__ddiv_rn(e, s), s);
+                    break;
                 case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
                 default: feas = (s >= thr_pl); key = e; break;             // PL_x
             }
@@ -180,7 +187,36 @@ __device__ __forceinline__ void finish_tile(const SweepArgs& a, const double* mS
         }
         __syncwarp();
         if (a.mode == kModeSweep)
-            select_row_warp(oS, oE, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
+            select_row_warp(oS, oE, nullptr, nullptr, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
+    }
+}
+
+// finish_tile for the four-model variant: mv[m] / sv[m] ([nk][n_f]) for models m < 4 (mv[m] null
+// when absent); direct EDP / ED2P predictions become the MIN_EDP / MIN_ED2P keys.
+__device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* mv, float* const* sv,
+                                             int nk, long long k0) {
+    const int n_f = a.n_f;
+    const int lane = threadIdx.x & 31;
+    const int nw = blockDim.x >> 5;
+    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
+        const long long k = k0 + kl;
+        for (int m = 0; m < 4; ++m) {
+            if (!mv[m]) continue;
+            const double* r = mv[m] + (size_t)kl * n_f;
+            float* o = sv[m] + (size_t)kl * n_f;
+            float* g = m == 0 ? a.S_out : m == 1 ? a.E_out : a.X_out[m - 2];
+            const double dv = a.def >= 0 ? r[a.def] : 1.0;
+            for (int i = lane; i < n_f; i += 32) {
+                const float v = a.def >= 0 ? __double2float_rn(__ddiv_rn(r[i], dv)) : __double2float_rn(r[i]);
+                o[i] = v;
+                if (g) g[k * n_f + i] = v;
+            }
+        }
+        __syncwarp();
+        if (a.mode == kModeSweep)
+            select_row_warp(sv[0] + (size_t)kl * n_f, sv[1] + (size_t)kl * n_f,
+                            mv[2] ? sv[2] + (size_t)kl * n_f : nullptr, mv[3] ? sv[3] + (size_t)kl * n_f : nullptr,
+                            n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
     }
 }
 
@@ -246,7 +282,7 @@ __global__ void __launch_bounds__(256) k_select(const __grid_constant__ SelectAr
     const int lane = threadIdx.x & 31;
     const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
     for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < a.n_k; k += warps) {
-        select_row_warp(a.S + k * a.n_f, a.E + k * a.n_f, a.n_f, a.def, a.n_t, a.kind, a.x,
+        select_row_warp(a.S + k * a.n_f, a.E + k * a.n_f, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.x,
                         a.choice + k * a.n_t, lane);
     }
 }

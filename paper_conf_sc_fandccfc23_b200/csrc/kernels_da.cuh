@@ -18,10 +18,11 @@
 // reaches, exactly.  Then forest = (double)acc * 2^-s / T, linear member, default-clock
 // normalisation and per-target argmin (finish_tile) as everywhere else.
 //
-// The kernel is bound by the L1 wavefront rate of the scattered block loads.  Every restart walk
-// of a task re-traverses the top of the same tree, so at task start each thread stages the root
-// block and its four grandchild blocks (the top two block levels, 160 B) in shared memory and the
-// walks read levels 0-1 from there (TOPC; about a quarter fewer global block loads per task).
+// The kernel is bound by the L1 wavefront rate of the scattered block loads and lives on L1 hits of
+// the upper tree blocks, which every restart walk re-reads; shared memory is kept small so L1 stays
+// large.  Optional TOPC (SYNERGY_TOPC=1) instead stages each task's top two block levels (root + 4
+// grandchild blocks, 160 B per thread) in shared memory: measured slower on B200 (round 1) because
+// the extra 20 KB per CTA comes out of L1.
 #pragma once
 #include "kernels_ws.cuh"
 
@@ -40,19 +41,29 @@ __device__ __forceinline__ uint4 lds_blk(unsigned a) {
     return v;
 }
 
+// Model m of the call: 0 speedup, 1 energy, 2 direct EDP, 3 direct ED2P (four-model variant).
+__device__ __forceinline__ const DevModel& da_model(const SweepArgs& a, int m) {
+    return m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+}
+
+__device__ __forceinline__ int da_trees(const SweepArgs& a, int m) {
+    if (m >= 2 && !a.has_x[m - 2]) return 0;
+    const DevModel& d = da_model(a, m);
+    return d.forest_weight != 0.0 ? d.n_trees : 0;
+}
+
 template <int NT, bool TOPC>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constant__ SweepArgs a) {
     extern __shared__ __align__(16) unsigned char smem[];
     const int n_f = a.n_f, F = a.F, XS = a.xs, KPC = a.tile_k;
+    const int NM = (a.has_x[0] || a.has_x[1]) ? 4 : 2;                      // models in this call
     const long long k0 = (long long)blockIdx.x * KPC;
     const int nk = (int)min((long long)KPC, a.n_k - k0);
-    long long* D = reinterpret_cast<long long*>(smem);                      // [KPC][2][n_f + 1]
-    long long* first = D + (size_t)KPC * 2 * (n_f + 1);                    // [NT][KPC][2]
-    double* mS = reinterpret_cast<double*>(first + (size_t)NT * KPC * 2);   // [KPC][n_f]
-    double* mE = mS + (size_t)KPC * n_f;
-    float* sS = reinterpret_cast<float*>(mE + (size_t)KPC * n_f);
-    float* sE = sS + (size_t)KPC * n_f;
-    float* fr = sE + (size_t)KPC * n_f;
+    long long* D = reinterpret_cast<long long*>(smem);                      // [KPC][NM][n_f + 1]
+    long long* first = D + (size_t)KPC * NM * (n_f + 1);                   // [NT][KPC][NM]
+    double* mv0 = reinterpret_cast<double*>(first + (size_t)NT * KPC * NM); // [NM][KPC][n_f]
+    float* sv0 = reinterpret_cast<float*>(mv0 + (size_t)NM * KPC * n_f);    // [NM][KPC][n_f]
+    float* fr = sv0 + (size_t)NM * KPC * n_f;
     float* xk = fr + n_f;                                                   // [KPC][XS]
     unsigned short* grid = reinterpret_cast<unsigned short*>(xk + KPC * XS);   // [kGrid + 2]
     int* counter = reinterpret_cast<int*>(grid + kGrid + 2);
@@ -71,9 +82,9 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
     if (threadIdx.x == 0) *counter = 0;
     for (int i = threadIdx.x; i < n_f; i += NT) fr[i] = __ldg(a.freqs + i);
     for (int b = threadIdx.x; b <= kGrid; b += NT) grid[b] = __ldg(a.grid + b);
-    for (int i = threadIdx.x; i < KPC * 2 * (n_f + 1); i += NT) D[i] = 0;
-    long long* myfirst = first + (size_t)threadIdx.x * KPC * 2;
-    for (int i = 0; i < KPC * 2; ++i) myfirst[i] = 0;
+    for (int i = threadIdx.x; i < KPC * NM * (n_f + 1); i += NT) D[i] = 0;
+    long long* myfirst = first + (size_t)threadIdx.x * KPC * NM;
+    for (int i = 0; i < KPC * NM; ++i) myfirst[i] = 0;
     __syncthreads();
 
     const int lane = threadIdx.x & 31;
@@ -82,20 +93,24 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
     const unsigned topc_a = su32(topc) + (unsigned)threadIdx.x * 160u;
     const float f0 = a.f0, inv_step = a.inv_step;
     const float f_last = fr[n_f - 1];
-    const int TS = a.ms.forest_weight != 0.0 ? a.ms.n_trees : 0;
-    const int TE = a.me.forest_weight != 0.0 ? a.me.n_trees : 0;
-    const int TT = TS + TE;
-    const int n_tasks = nk * TT;
-    const int BD = max(TS ? a.ms.bdepth : 1, TE ? a.me.bdepth : 1);
-    const uint4* __restrict__ bS = a.ms.blocks;
-    const uint4* __restrict__ bE = a.me.blocks;
+    // tasks of one kernel: the trees of model 0, then 1, 2, 3 (cumulative counts c1 < c2 < c3 < TT)
+    const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = NM > 2 ? da_trees(a, 2) : 0,
+              T3 = NM > 2 ? da_trees(a, 3) : 0;
+    const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
+    // a task is (kernel, model, tree, clock sub-range r of R): small batches split each tree's
+    // clock axis so more lanes share the walks (order-free sums make the pieces independent)
+    const int R = max(1, a.nsub);
+    const int n_tasks = nk * TT * R;
+    int BD = 1;
+    for (int m = 0; m < NM; ++m)
+        if (da_trees(a, m)) BD = max(BD, da_model(a, m).bdepth);
 
     long long vprev = 0;
     int task = -1;                      // -1: idle
-    int kl = 0;
-    bool isE = false;
+    int kl = 0, mi = 0, ra = 0, rb = n_f;   // sub-range [ra, rb) of the clock axis
     double scale = 1.0;
     int root = 0, lo = 0;
+    const uint4* own = a.ms.blocks;
     unsigned xrow_a = xk_a;
     float f_lo = 0.0f, tmin = CUDART_INF_F;
     bool exhausted = false;
@@ -112,16 +127,20 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
                 const int j = base + __popc(need & lm_lt);
                 if (j < n_tasks) {
                     task = j;
-                    kl = j / TT;
-                    const int jj = j - kl * TT;
-                    isE = jj >= TS;
-                    const DevModel& m = isE ? a.me : a.ms;
+                    kl = j / (TT * R);
+                    const int rem = j - kl * TT * R;
+                    const int jj = rem / R, r = rem - jj * R;
+                    ra = (int)(((long long)r * n_f) / R);
+                    rb = (int)(((long long)(r + 1) * n_f) / R);
+                    mi = jj < c1 ? 0 : jj < c2 ? 1 : jj < c3 ? 2 : 3;
+                    const int tree = jj - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3);
+                    const DevModel& m = da_model(a, mi);
                     scale = m.fx_scale;
-                    root = __ldg(m.broot + (isE ? jj - TS : jj));
+                    own = m.blocks;
+                    root = __ldg(m.broot + tree);
                     xrow_a = xk_a + 4u * (unsigned)(kl * XS);
                     if (TOPC) {                               // stage the top two block levels
-                        const uint4* bl = isE ? bE : bS;
-                        const uint4 A0 = ldg_blk(bl + 2 * (size_t)root), B0 = ldg_blk(bl + 2 * (size_t)root + 1);
+                        const uint4 A0 = ldg_blk(own + 2 * (size_t)root), B0 = ldg_blk(own + 2 * (size_t)root + 1);
                         sts_blk(topc_a, A0);
                         sts_blk(topc_a + 16u, B0);
                         const unsigned cw = A0.w;
@@ -131,25 +150,25 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
                             const bool inner = (int)(cw & 0xffu) <= F && (int)((cw >> (8 + 8 * (s2 >> 1))) & 0xffu) <= F &&
                                                !((cw >> (24 + s2)) & 1u);
                             if (inner) {
-                                sts_blk(topc_a + 32u * (1 + s2), ldg_blk(bl + 2 * (size_t)gs[s2]));
-                                sts_blk(topc_a + 32u * (1 + s2) + 16u, ldg_blk(bl + 2 * (size_t)gs[s2] + 1));
+                                sts_blk(topc_a + 32u * (1 + s2), ldg_blk(own + 2 * (size_t)gs[s2]));
+                                sts_blk(topc_a + 32u * (1 + s2) + 16u, ldg_blk(own + 2 * (size_t)gs[s2] + 1));
                             }
                         }
                     }
-                    lo = 0;
-                    f_lo = lds_f(fr_a);
+                    lo = ra;
+                    f_lo = lds_f(fr_a + 4u * (unsigned)min(ra, n_f - 1));
                     tmin = CUDART_INF_F;
+                    if (ra >= rb) task = -1;                  // empty sub-range (R > n_f)
                 } else {
                     exhausted = true;
                 }
             }
         }
         if (!__any_sync(0xffffffffu, task >= 0)) break;
-        // one restart walk per busy lane, lockstep over BD lane-paired block steps
+        // one restart walk per busy lane, lockstep over BD 2-level block steps
         float leaf = 0.0f;
         int bk = root;
         bool done = task < 0;
-        const uint4* __restrict__ own = isE ? bE : bS;
         if (TOPC) {                                   // levels 0-1 from the shared cache
             int gs = 0;
             if (!done) block_decide(lds_blk(topc_a), lds_blk(topc_a + 16u), bk, gs, done, leaf, tmin, f_lo, xrow_a, F);
@@ -168,10 +187,12 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
         if (task >= 0) {
             const int hi = (tmin < f_last) ? clock_cut_s(fr_a, grid_a, f0, inv_step, tmin, lo, n_f) : n_f;
             const long long v = __double2ll_rn(__dmul_rn((double)leaf, scale));   // exact
-            if (lo == 0) myfirst[kl * 2 + (isE ? 1 : 0)] += v;                    // thread-private
-            else atomic_add_s64(D + ((size_t)kl * 2 + (isE ? 1 : 0)) * (n_f + 1) + lo, v - vprev);
+            long long* Drow = D + ((size_t)kl * NM + mi) * (n_f + 1);
+            if (lo == 0) myfirst[kl * NM + mi] += v;                               // thread-private
+            else atomic_add_s64(Drow + lo, lo == ra ? v : v - vprev);             // sub-range start: +v
             vprev = v;
-            if (hi >= n_f) {
+            if (hi >= rb) {                                                        // run reaches the range end
+                if (rb < n_f) atomic_add_s64(Drow + rb, -v);
                 task = -1;
             } else {
                 lo = hi;
@@ -184,17 +205,18 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
 
     // fold the thread-private first-run sums into D[.][.][0], then prefix sums over clocks
     const int warp = threadIdx.x >> 5, nw = NT / 32;
-    for (int p = warp; p < 2 * nk; p += nw) {            // p = kernel * 2 + model
+    for (int p = warp; p < NM * nk; p += nw) {            // p = kernel * NM + model
+        const int pk = p / NM, pm = p - pk * NM;
+        if (pm >= 2 && !a.has_x[pm - 2]) continue;
         long long s = 0;
-        for (int t2 = lane; t2 < NT; t2 += 32) s += first[(size_t)t2 * KPC * 2 + p];
+        for (int t2 = lane; t2 < NT; t2 += 32) s += first[(size_t)t2 * KPC * NM + p];
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
         long long* Dm = D + (size_t)p * (n_f + 1);
         if (lane == 0) Dm[0] += s;
         __syncwarp();
-        const int pk = p >> 1, pm = p & 1;
-        const DevModel& m = pm ? a.me : a.ms;
-        double* out = (pm ? mE : mS) + (size_t)pk * n_f;
+        const DevModel& m = da_model(a, pm);
+        double* out = mv0 + ((size_t)pm * KPC + pk) * n_f;
         const float* xrow = xk + pk * XS;
         const int chunk = (n_f + 31) / 32;
         const int i0 = min(n_f, lane * chunk), i1 = min(n_f, i0 + chunk);
@@ -215,7 +237,14 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_sweep_da(const __grid_constan
         }
     }
     __syncthreads();
-    finish_tile(a, mS, mE, sS, sE, nk, k0);
+    double* mv[4];
+    float* sv[4];
+    for (int m = 0; m < 4; ++m) {
+        const bool present = m < 2 || (NM > 2 && a.has_x[m - 2]);
+        mv[m] = present ? mv0 + (size_t)m * KPC * n_f : nullptr;
+        sv[m] = present ? sv0 + (size_t)m * KPC * n_f : nullptr;
+    }
+    finish_tile4(a, mv, sv, nk, k0);
 }
 
 }  // namespace syn

@@ -259,20 +259,27 @@ cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaS
 // Difference-array kernel: KPC kernels per CTA, exact int64 leaf sums (needs fx_ok forests).
 // KPC grows when a kernel has fewer trees than the CTA has threads, so lanes keep walking and
 // the per-CTA staging / finish is amortised.
-size_t da_head(int nt, int kpc, int n_f, int xs) {
-    const size_t h = (size_t)kpc * 2 * (n_f + 1) * 8 + (size_t)nt * kpc * 2 * 8 + (size_t)kpc * n_f * 24 +
+size_t da_head(int nt, int kpc, int n_f, int xs, int nm) {
+    const size_t h = (size_t)kpc * nm * (n_f + 1) * 8 + (size_t)nt * kpc * nm * 8 + (size_t)nm * kpc * n_f * 12 +
                      (size_t)n_f * 4 + (size_t)kpc * xs * 4 + (size_t)(kGrid + 2) * 2 + 16;
     return (h + 15) & ~(size_t)15;
 }
 
-size_t da_smem(int nt, int kpc, int n_f, int xs) {
-    return da_head(nt, kpc, n_f, xs) + (size_t)nt * 160;   // + per-thread top-block cache
+// The per-thread top-block cache (TOPC) is only allocated when enabled: shared memory comes out of
+// the same 256 KB as L1, and this kernel lives on L1 hits of the upper tree blocks.
+bool da_topc() { return env_int("SYNERGY_TOPC", 0) != 0; }
+
+size_t da_smem(int nt, int kpc, int n_f, int xs, int nm) {
+    return da_head(nt, kpc, n_f, xs, nm) + (da_topc() ? (size_t)nt * 160 : 0);
 }
 
-bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c) {
+bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c,
+               const syn_model* x2 = nullptr, const syn_model* x3 = nullptr) {
     if (n_f > 2048) return false;
     if ((sp->n_trees && !sp->dm.fx_ok) || (en->n_trees && !en->dm.fx_ok)) return false;
-    const int tt = sp->n_trees + en->n_trees;
+    if ((x2 && x2->n_trees && !x2->dm.fx_ok) || (x3 && x3->n_trees && !x3->dm.fx_ok)) return false;
+    const int nm = (x2 || x3) ? 4 : 2;
+    const int tt = std::max(1, sp->n_trees + en->n_trees + (x2 ? x2->n_trees : 0) + (x3 ? x3->n_trees : 0));
     int nt = env_int("SYNERGY_NT", 128);
     nt = nt >= 256 ? 256 : (nt >= 128 ? 128 : 64);
     int kpc = tt >= nt ? 1 : (3 * nt + 2 * tt - 1) / (2 * tt);      // ~1.5 tasks per thread
@@ -280,15 +287,21 @@ bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f,
     kpc = env_int("SYNERGY_KPC", kpc);
     kpc = (int)std::max<long long>(1, std::min<long long>(std::min(kpc, 16), std::max<long long>(n_k, 1)));
     c.algo = 3;
-    c.slots = c.tilp = 0;
+    c.tilp = 0;
     c.tile_k = kpc;
     c.nt = nt;
     c.xs = (F + 2) | 1;
     c.tc = c.words = c.vcap = c.vs = c.region = 0;
     c.win = c.slot_bytes = c.head_bytes = 0;
-    c.smem = da_smem(nt, kpc, n_f, c.xs);
-    while (c.smem > 200 * 1024 && c.tile_k > 1) c.smem = da_smem(nt, --c.tile_k, n_f, c.xs);
-    c.head_bytes = (int)da_head(nt, c.tile_k, n_f, c.xs);
+    // small batches: split each (kernel, tree) task into R clock sub-ranges so that there are at
+    // least ~4 tasks per resident lane (R = 1 for large batches: every split costs an extra walk)
+    const long long lanes = (long long)sm_count(0) * 1024, tasks = std::max<long long>(1, n_k * tt);
+    int nsub = (int)std::min<long long>(4, std::max<long long>(1, (4 * lanes + tasks - 1) / tasks));
+    nsub = std::max(1, std::min(env_int("SYNERGY_NSUB", nsub), std::max(1, n_f)));
+    c.slots = nsub;                                        // carried to SweepArgs.nsub
+    c.smem = da_smem(nt, kpc, n_f, c.xs, nm);
+    while (c.smem > 200 * 1024 && c.tile_k > 1) c.smem = da_smem(nt, --c.tile_k, n_f, c.xs, nm);
+    c.head_bytes = (int)da_head(nt, c.tile_k, n_f, c.xs, nm);
     return c.smem <= 200 * 1024;
 }
 
@@ -305,7 +318,7 @@ cudaError_t launch_da_t(const SweepArgs& a, const Config& c, long long grid, cud
 }
 
 cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    const bool topc = env_int("SYNERGY_TOPC", 1) != 0;
+    const bool topc = da_topc();
     if (c.nt == 256) return topc ? launch_da_t<256, true>(a, c, grid, st) : launch_da_t<256, false>(a, c, grid, st);
     if (c.nt == 128) return topc ? launch_da_t<128, true>(a, c, grid, st) : launch_da_t<128, false>(a, c, grid, st);
     return topc ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
@@ -416,6 +429,7 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     a.grid = clocks->d_grid;
     a.f0 = clocks->f0;
     a.inv_step = clocks->inv_step;
+    a.nsub = c.algo == 3 ? c.slots : 1;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
     cudaError_t e = c.algo == 3 ? launch_da(a, c, grid, st)
@@ -741,6 +755,72 @@ syn_status synergy_sweep(const syn_model* sp, const syn_model* en, const float* 
                          int32_t n_t, int32_t* d_choice, float* d_S, float* d_E, syn_stream stream) {
     return run_sweep(sp, en, d_features, n_k, F, clocks, def, targets, n_t, d_choice, d_S, d_E, kModeSweep,
                      static_cast<cudaStream_t>(stream));
+}
+
+syn_status synergy_sweep4(const syn_model* const* models, const float* d_features, int64_t n_k, int32_t F,
+                          const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
+                          int32_t* d_choice, float* d_pred, syn_stream stream) {
+    if (!models) return fail(SYN_ERR_INVALID_ARG, "models is NULL");
+    const syn_model* sp = models[0];
+    const syn_model* en = models[1];
+    const syn_model* x2 = models[2];
+    const syn_model* x3 = models[3];
+    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, kModeSweep);
+    if (vs != SYN_OK) return vs;
+    for (const syn_model* xm : {x2, x3}) {
+        if (!xm) continue;
+        if (xm->n_inputs != F + 1) return fail(SYN_ERR_INVALID_ARG, "direct EDP/ED2P model n_inputs mismatch");
+        if (xm->device != clocks->device) return fail(SYN_ERR_INVALID_ARG, "model device differs from clocks");
+    }
+    if (n_k == 0) {
+        g_last = {0, 0, 0, 0, 0};
+        return ok();
+    }
+    if (!d_features || !d_choice) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    const int n_f = clocks->n_f;
+    Config c;
+    if (!choose_da(sp, en, n_k, n_f, F, c, x2, x3))
+        return fail(SYN_ERR_UNSUPPORTED, "four-model sweep needs forests within the exact int64 leaf range and n_freqs <= 2048");
+    SweepArgs a;
+    memset(&a, 0, sizeof a);
+    a.ms = sp->dm;
+    a.me = en->dm;
+    if (x2) { a.mx[0] = x2->dm; a.has_x[0] = 1; }
+    if (x3) { a.mx[1] = x3->dm; a.has_x[1] = 1; }
+    if (!x2 && !x3) a.has_x[0] = 0;
+    a.features = d_features;
+    a.n_k = n_k;
+    a.F = F;
+    a.freqs = clocks->d_freqs;
+    a.n_f = n_f;
+    a.def = def;
+    a.n_t = n_t;
+    for (int t = 0; t < n_t; ++t) {
+        a.kind[t] = targets[t].kind;
+        a.x[t] = targets[t].x;
+    }
+    a.choice = d_choice;
+    if (d_pred) {
+        const size_t plane = (size_t)n_k * n_f;
+        a.S_out = d_pred;
+        a.E_out = d_pred + plane;
+        a.X_out[0] = x2 ? d_pred + 2 * plane : nullptr;
+        a.X_out[1] = x3 ? d_pred + 3 * plane : nullptr;
+    }
+    a.mode = kModeSweep;
+    a.tile_k = c.tile_k;
+    a.xs = c.xs;
+    a.head_bytes = c.head_bytes;
+    a.grid = clocks->d_grid;
+    a.f0 = clocks->f0;
+    a.inv_step = clocks->inv_step;
+    a.nsub = c.slots;
+    const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
+    if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
+    cudaError_t e = launch_da(a, c, grid, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "k_sweep_da launch");
+    g_last = {1, n_k * (long long)n_f, grid, c.nt, 3000 + c.tile_k};
+    return ok();
 }
 
 syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32_t n_f, int32_t def,

@@ -71,6 +71,7 @@ def load(path: str = LIB_PATH) -> C.CDLL:
         "synergy_predict": (I32, [P, P, P, I64, I32, P, I32, P, P, P]),
         "synergy_select": (I32, [P, P, I64, I32, I32, P, I32, P, P]),
         "synergy_sweep": (I32, [P, P, P, I64, I32, P, I32, P, I32, P, P, P, P]),
+        "synergy_sweep4": (I32, [P, P, I64, I32, P, I32, P, I32, P, P, P]),
         "synergy_workspace_create": (I32, [I32, P]),
         "synergy_workspace_destroy": (I32, [P]),
         "synergy_sweep_host": (I32, [P, P, P, P, I64, I32, P, I32, P, I32, P, P]),
@@ -234,6 +235,23 @@ def sweep(speedup: Model, energy: Model, features, clocks: Clocks, default_idx: 
                                 _dev_ptr(out_speedup, torch.float32, (n_k, clocks.n), "out_speedup"),
                                 _dev_ptr(out_energy, torch.float32, (n_k, clocks.n), "out_energy"),
                                 _stream(stream)))
+    return out
+
+
+def sweep4(models, features, clocks: Clocks, default_idx: int, targets, out=None, out_pred=None, stream=None):
+    """synergy_sweep4: four-model variant, models = [speedup, energy, edp|None, ed2p|None];
+    out_pred (optional) = float32 [4][n_k][n_f] normalised predictions."""
+    import torch
+    n_k, F = features.shape
+    tg, n_t = _targets(targets)
+    if out is None:
+        out = torch.empty((n_k, n_t), dtype=torch.int32, device=features.device)
+    handles = (C.c_void_p * 4)(*[None if m is None else m.handle.value for m in models])
+    _check(load().synergy_sweep4(handles, _dev_ptr(features, torch.float32, name="features"), n_k, F,
+                                 clocks.handle, int(default_idx), tg, n_t,
+                                 _dev_ptr(out, torch.int32, (n_k, n_t), "out"),
+                                 _dev_ptr(out_pred, torch.float32, (4, n_k, clocks.n), "out_pred"),
+                                 _stream(stream)))
     return out
 
 

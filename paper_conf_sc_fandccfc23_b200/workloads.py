@@ -270,7 +270,12 @@ def _complete_trees(rng, n_trees, depth, F, freqs, dvfs: _DVFS, which: str, p_fr
     centre = 0.5 * (lo + np.minimum(hi, 1024.0))
     beta = dvfs.beta(centre)
     fc = 0.5 * (fr[np.clip(ilo, 0, nf - 1)] + fr[np.clip(ihi, 0, nf - 1)])
-    y = dvfs.speedup(beta, fc) if which == "speedup" else dvfs.energy(beta, fc)
+    if which == "speedup":
+        y = dvfs.speedup(beta, fc)
+    elif which == "edp":                          # E * T, T = 1/S
+        y = dvfs.energy(beta, fc) / dvfs.speedup(beta, fc)
+    else:
+        y = dvfs.energy(beta, fc)
     y = y + rng.normal(0.0, noise, size=y.shape)
     value[:, first:] = np.clip(y, 0.25, np.nextafter(np.float32(4.0), np.float32(0.0))).astype(np.float32)
     # children arrays
@@ -310,6 +315,18 @@ def linear_speedup_model(seed_seq, F, freqs, def_idx) -> ModelSpec:
     return ModelSpec(n_inputs=F + 1, linear_weight=1.0, lin_w=w, lin_b=b)
 
 
+def linear_ed2p_model(seed_seq, F, freqs, def_idx) -> ModelSpec:
+    """Linear ED2P regressor (Table 2 "Best" for MIN_ED2P: Linear): ED2P = E*T^2 falls with the
+    clock on compute-bound kernels; negative clock weight, b so ED2P(f_def) ~ 1 and > 0."""
+    rng = np.random.Generator(np.random.PCG64(seed_seq))
+    f_def, f_max = float(freqs[def_idx]), float(freqs[-1])
+    w = np.zeros(F + 1)
+    w[:F] = rng.normal(0.0, 1e-5, size=F)
+    w[F] = -rng.uniform(0.3, 0.6) / f_max
+    b = 1.0 - w[F] * f_def - float(np.sum(w[:F]) * 100.0)
+    return ModelSpec(n_inputs=F + 1, linear_weight=1.0, lin_w=w, lin_b=b)
+
+
 # ------------------------------------------------------------------------ configs
 
 CONFIGS = {
@@ -344,6 +361,22 @@ def make_models(cfg: str):
     d = default_index(freqs)
     return (_model(sp, sp_ss, N_STATIC, freqs, d, "speedup"),
             _model(en, en_ss, N_STATIC, freqs, d, "energy"), freqs, d)
+
+
+def make_models4(cfg: str = "c2"):
+    """Four-model variant on config cfg's shapes, each target's
+    model family from Table 2's "Best" column (L403-L412): speedup Linear (MAX_PERF, PL), energy
+    RandomForest (MIN_ENERGY, ES), EDP RandomForest (MIN_EDP), ED2P Linear (MIN_ED2P)."""
+    n_k, n_f, sp, en, tg = CONFIGS[cfg]
+    ss = np.random.SeedSequence(SEED_BASE + 100 + CONFIG_INDEX[cfg])
+    s_sp, s_en, s_edp, s_ed2p = ss.spawn(4)
+    freqs = clock_table(n_f)
+    d = default_index(freqs)
+    T, D = (en[1], en[2]) if en[0] == "rf" else (100, 12)
+    return ([linear_speedup_model(s_sp, N_STATIC, freqs, d),
+             forest_model(s_en, T, D, N_STATIC, freqs, d, "energy"),
+             forest_model(s_edp, T, D, N_STATIC, freqs, d, "edp"),
+             linear_ed2p_model(s_ed2p, N_STATIC, freqs, d)], freqs, d)
 
 
 def make_features(cfg: str, row0: int = 0, n: Optional[int] = None) -> np.ndarray:

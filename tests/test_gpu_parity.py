@@ -26,7 +26,9 @@ def _build():
 #   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
 #   da_nt256  k_sweep_da with 256 threads per CTA
 #   da_kpc5   k_sweep_da with 5 kernels per CTA (tasks of several kernels per warp, ragged tile)
-#   da_notopc k_sweep_da without the shared top-block cache, 3 kernels per CTA
+#   da_nsub3  k_sweep_da splitting every (kernel, tree) task into 3 clock sub-ranges
+#   da_nsub64 k_sweep_da with 64 sub-ranges (single-clock and empty ranges on small tables)
+#   da_topc   k_sweep_da with the shared top-block cache (TOPC), 3 kernels per CTA
 #   ws        in-order warp-streaming kernel (k_sweep_ws), 2 kernels per CTA, window 64
 #   ws_tight  k_sweep_ws with window 32 (= warp width: refills wait on the oldest tree), 1 run
 #             value kept per tree (every later run takes the direct-walk fallback), 3 kernels/CTA
@@ -37,7 +39,7 @@ def _build():
 #   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
 VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERGY_NT": "256"},
-            "da_kpc5": {"SYNERGY_KPC": "5"}, "da_notopc": {"SYNERGY_TOPC": "0", "SYNERGY_KPC": "3"},
+            "da_kpc5": {"SYNERGY_KPC": "5"}, "da_nsub3": {"SYNERGY_NSUB": "3"}, "da_nsub64": {"SYNERGY_NSUB": "64", "SYNERGY_KPC": "2"}, "da_topc": {"SYNERGY_TOPC": "1", "SYNERGY_KPC": "3"},
             "ws": {"SYNERGY_ALGO": "ws"},
             "ws_tight": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"},
             "ws_wide": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
@@ -45,7 +47,7 @@ VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERG
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC")
+KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
@@ -153,6 +155,53 @@ def test_out_of_range_leaves_fall_back_to_ordered_kernel():
     assert syn.last_launch()["variant"] // 1000 != 3
     assert_bits_equal(S, rS, "raw S")
     assert_bits_equal(E, rE, "raw E")
+
+
+def _gpu_sweep4(models, feats, freqs, d, targets):
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    hm = [None if m is None else syn.Model(m) for m in models]
+    ck = syn.Clocks(freqs)
+    f = torch.from_numpy(np.ascontiguousarray(feats)).cuda()
+    P = torch.full((4, f.shape[0], len(freqs)), -7.0, dtype=torch.float32, device="cuda")
+    ch = syn.sweep4(hm, f, ck, d, targets, out_pred=P)
+    torch.cuda.synchronize()
+    return ch.cpu().numpy(), P.cpu().numpy()
+
+
+@pytest.mark.parametrize("cfg", ["c1", "c2"])
+def test_four_model_variant_bit_exact(cfg, variant):
+    """NEXT f1: speedup + energy + direct EDP (RF) + direct ED2P (linear)."""
+    if VARIANTS[variant].get("SYNERGY_ALGO"):
+        pytest.skip("four-model sweep always runs on k_sweep_da")
+    models, freqs, d = W.make_models4(cfg)
+    feats = W.make_features(cfg)
+    targets = W.targets_six()
+    ref = oracle.sweep4(models, feats, freqs, d, targets, want_pred=True)
+    ch, P = _gpu_sweep4(models, feats, freqs, d, targets)
+    for m in range(4):
+        assert_bits_equal(P[m], ref["P"][m], f"model {m}")
+    assert_choices(ch, ref["choice"])
+
+
+def test_four_model_variant_lookup_tables_and_missing_models():
+    """Per-clock lookup-table EDP/ED2P trees (MIN_EDP / MIN_ED2P = first argmin of the tables) and
+    one absent direct model (derived key) against the oracle."""
+    from test_oracle_four_models import lookup_tree
+    w = W.make_config("c1")
+    rng = np.random.default_rng(12)
+    edp = rng.integers(1, 9, size=w.n_freqs).astype(np.float32) / 4
+    edp[3] = -1.0
+    ed2p = rng.integers(1, 9, size=w.n_freqs).astype(np.float32) / 4
+    for models in ([w.speedup, w.energy, lookup_tree(w.freqs, edp, w.n_features), lookup_tree(w.freqs, ed2p, w.n_features)],
+                   [w.speedup, w.energy, None, lookup_tree(w.freqs, ed2p, w.n_features)],
+                   [w.speedup, w.energy, None, None]):
+        ref = oracle.sweep4(models, w.features, w.freqs, w.default_idx, w.targets, want_pred=True)
+        ch, P = _gpu_sweep4(models, w.features, w.freqs, w.default_idx, w.targets)
+        assert_choices(ch, ref["choice"])
+        for m in range(4):
+            if models[m] is not None:
+                assert_bits_equal(P[m], ref["P"][m], f"model {m}")
 
 
 def test_empty_batch_is_noop():
