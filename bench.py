@@ -195,12 +195,16 @@ def oracle_single_core(cfg, n_k_cap, budget_s=10.0):
     return evals / el, evals, el
 
 
-def run_walk_work(cfg, row0, n_rows, cap=1000):
-    """Run-walk work of the launched rows, counted by the oracle on the first min(n_rows, cap)
-    rows (exact when n_rows <= cap): runs of clocks sharing a leaf and their 2-level block fetches."""
+def run_walk_work(cfg, row0, n_rows, budget=5e8):
+    """Run-walk work of the launched rows, counted by the oracle on the first rows that fit a
+    budget of ~5e8 node decisions (all rows for c1/c2/c5): runs of clocks sharing a leaf and their
+    2-level block fetches."""
     import oracle
     from paper_conf_sc_fandccfc23_b200 import workloads as W
-    n = min(n_rows, cap)
+    n_f = W.CONFIGS[cfg][1]
+    sp, en = W.make_models(cfg)[:2]
+    per_row = max(1, n_f * (decisions_per_eval(sp) + decisions_per_eval(en)))
+    n = int(min(n_rows, max(16, budget // per_row)))
     if n == 0:
         return None
     w = W.make_config(cfg, row0=row0, n=n)

@@ -166,6 +166,35 @@ syn_status synergy_sweep4(const syn_model *const *models, const float *d_feature
                           const syn_target *h_targets, int32_t n_targets, int32_t *d_choice,
                           float *d_pred, syn_stream stream);
 
+/* Frequency plan emission ("the predicted frequency configuration is made available
+ * to the SYCL library at runtime"; L187 q.submit(MIN_EDP, ...)): d_mhz[k][t] = f[d_choice[k][t]]
+ * in MHz, NaN where the choice is -1 (or out of range).  Applying clocks needs privileged NVML
+ * access (L330, L342), so the library only emits the plan.  INVALID_ARG: null buffers,
+ * n_kernels < 0, n_targets outside [1, SYNERGY_MAX_TARGETS]. */
+syn_status synergy_plan(const int32_t *d_choice, int64_t n_kernels, int32_t n_targets,
+                        const syn_clocks *clocks, float *d_mhz, syn_stream stream);
+
+/* Pareto front per kernel ("the red line is the Pareto front", L247, L374):
+ * d_front[k][i] = 1 iff clock i is a valid candidate (S, E finite and > 0) and no valid clock j
+ * has S_j >= S_i and E_j <= E_i with one strict, else 0.  Inputs as synergy_select.
+ * INVALID_ARG: null buffers, n_kernels < 0, n_freqs outside [1, SYNERGY_MAX_FREQS]. */
+syn_status synergy_pareto(const float *d_speedup, const float *d_energy, int64_t n_kernels,
+                          int32_t n_freqs, uint8_t *d_front, syn_stream stream);
+
+/* Frequency-choice error (Table 2: APE / MAPE / RMSE "between the predicted and
+ * actual optimal frequency"): per kernel and target, the target's objective on the ground-truth
+ * table (d_speedup_true, d_energy_true) at the predicted clock d_choice_pred[k][t] vs at the
+ * actual optimal clock (the target selected on the ground truth, as synergy_select).  Objective:
+ * MAX_PERF, ES_x -> S; MIN_ENERGY, PL_x -> E; MIN_EDP -> E/S; MIN_ED2P -> (E/S)/S (fp64).
+ * d_err[k][t] = {APE, predicted - actual} (NaN, NaN where either clock is -1);
+ * d_summary[t] = {MAPE, RMSE, kernels counted} over the counted kernels (fp64, fixed-order
+ * reduction).  Errors as synergy_select plus null d_choice_pred / d_err / d_summary. */
+syn_status synergy_choice_error(const float *d_speedup_true, const float *d_energy_true,
+                                int64_t n_kernels, int32_t n_freqs, int32_t default_idx,
+                                const syn_target *h_targets, int32_t n_targets,
+                                const int32_t *d_choice_pred, double *d_err, double *d_summary,
+                                syn_stream stream);
+
 /* End-to-end host-buffer path: copies h_features host->device into the workspace, runs
  * synergy_sweep, copies the choices device->host into h_choice, all enqueued on `stream`
  * (h_choice is valid after the stream is synchronised; pinned host buffers make the copies

@@ -56,6 +56,11 @@ def _load():
         lib.oracle_select.restype = C.c_int
         lib.oracle_select.argtypes = [P, P, C.c_int64, C.c_int32, C.c_int32, P, P, C.c_int32,
                                       P, P]
+        lib.oracle_pareto.restype = C.c_int
+        lib.oracle_pareto.argtypes = [P, P, C.c_int64, C.c_int32, P]
+        lib.oracle_choice_error.restype = C.c_int
+        lib.oracle_choice_error.argtypes = [P, P, C.c_int64, C.c_int32, C.c_int32, P, P, C.c_int32, P, P, P,
+                                            P, P]
         lib.oracle_sweep4.restype = C.c_int
         lib.oracle_sweep4.argtypes = [P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32, P, P,
                                       C.c_int32, P, P]
@@ -212,6 +217,38 @@ def sweep4(models, features, freqs, default_idx, targets, want_pred=False):
     if rc != 0:
         raise OracleError("oracle_sweep4: invalid arguments")
     return {"choice": ch, "P": P} if want_pred else {"choice": ch}
+
+
+def pareto(S, E):
+    """uint8 front mask [n_k][n_f] of the (max S, min E) Pareto front per kernel."""
+    lib = _load()
+    S = np.ascontiguousarray(S, dtype=np.float32)
+    E = np.ascontiguousarray(E, dtype=np.float32)
+    if S.ndim == 1:
+        S, E = S[None], E[None]
+    front = np.empty(S.shape, np.uint8)
+    if lib.oracle_pareto(_ptr(S), _ptr(E), S.shape[0], S.shape[1], _ptr(front)) != 0:
+        raise OracleError("oracle_pareto: invalid arguments")
+    return front
+
+
+def choice_error(S_true, E_true, default_idx, targets, choice_pred):
+    """(ape [n_k][n_t], mape [n_t], rmse [n_t], counted [n_t]) of predicted choices vs truth."""
+    lib = _load()
+    S_true = np.ascontiguousarray(S_true, dtype=np.float32)
+    E_true = np.ascontiguousarray(E_true, dtype=np.float32)
+    choice_pred = np.ascontiguousarray(choice_pred, dtype=np.int32)
+    n_k, n_f = S_true.shape
+    kinds, xs = _targets(targets)
+    n_t = len(kinds)
+    ape = np.empty((n_k, n_t), np.float64)
+    mape = np.empty(n_t, np.float64)
+    rmse = np.empty(n_t, np.float64)
+    cnt = np.empty(n_t, np.int64)
+    if lib.oracle_choice_error(_ptr(S_true), _ptr(E_true), n_k, n_f, int(default_idx), _ptr(kinds), _ptr(xs),
+                               n_t, _ptr(choice_pred), _ptr(ape), _ptr(mape), _ptr(rmse), _ptr(cnt)) != 0:
+        raise OracleError("oracle_choice_error: invalid arguments")
+    return ape, mape, rmse, cnt
 
 
 def sweep_workload(w, **kw):

@@ -81,6 +81,17 @@ int oracle_sweep4(const oracle_model *const *models, const float *features, int6
                   int32_t n_features, const float *freqs, int32_t n_f, int32_t default_idx,
                   const int32_t *kind, const float *x, int32_t n_t, int32_t *choice, float *P);
 
+/* Pareto front per kernel: front[k][i] = 1 iff clock i is valid and not
+ * dominated in (max S, min E) by a valid clock. */
+int oracle_pareto(const float *S, const float *E, int64_t n_k, int32_t n_f, uint8_t *front);
+
+/* Frequency-choice error APE / MAPE / RMSE (Table 2) of predicted choices
+ * against the targets selected on a ground-truth table (S_true, E_true); ape nullable. */
+int oracle_choice_error(const float *S_true, const float *E_true, int64_t n_k, int32_t n_f,
+                        int32_t default_idx, const int32_t *kind, const float *x, int32_t n_t,
+                        const int32_t *choice_pred, double *ape, double *mape, double *rmse,
+                        int64_t *counted);
+
 #ifdef __cplusplus
 }
 #endif

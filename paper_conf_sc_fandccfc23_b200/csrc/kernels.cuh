@@ -287,4 +287,103 @@ __global__ void __launch_bounds__(256) k_select(const __grid_constant__ SelectAr
     }
 }
 
+// Pareto front: one warp per kernel, each lane tests its clocks against every clock of the row
+// (row read through L1; all lanes read the same j, so the loads are broadcasts).
+__global__ void __launch_bounds__(256) k_pareto(const float* __restrict__ S, const float* __restrict__ E,
+                                                long long n_k, int n_f, unsigned char* __restrict__ front) {
+    const int lane = threadIdx.x & 31;
+    const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+    for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < n_k; k += warps) {
+        const float* s = S + k * n_f;
+        const float* e = E + k * n_f;
+        for (int i0 = 0; i0 < n_f; i0 += 32) {
+            const int i = i0 + lane;
+            const float si = i < n_f ? __ldg(s + i) : 0.0f, ei = i < n_f ? __ldg(e + i) : 0.0f;
+            bool on = i < n_f && valid_pred(si, ei);
+            for (int j = 0; j < n_f; ++j) {
+                const float sj = __ldg(s + j), ej = __ldg(e + j);
+                if (valid_pred(sj, ej) && sj >= si && ej <= ei && (sj > si || ej < ei)) on = false;
+            }
+            if (i < n_f) front[k * n_f + i] = on ? 1 : 0;
+        }
+    }
+}
+
+__device__ __forceinline__ double target_objective(int kind, float s, float e) {
+    const double ds = (double)s, de = (double)e;
+    switch (kind) {
+        case 0: case 4: return ds;
+        case 1: case 5: return de;
+        case 2: return __ddiv_rn(de, ds);
+        default: return __ddiv_rn(__ddiv_rn(de, ds), ds);
+    }
+}
+
+// Choice error, per kernel (one warp): the truth's choice per target (select_row_warp on the
+// ground-truth row, into shared memory), then lane t computes target t's APE and difference.
+__global__ void __launch_bounds__(256) k_choice_error(const __grid_constant__ SelectArgs a,
+                                                      const int* __restrict__ pred, double* __restrict__ err) {
+    __shared__ int truth[8][kMaxTargets];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
+    for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + w; k < a.n_k; k += warps) {
+        const float* s = a.S + k * a.n_f;
+        const float* e = a.E + k * a.n_f;
+        select_row_warp(s, e, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.x, truth[w], lane);
+        __syncwarp();
+        if (lane < a.n_t) {
+            const int ip = __ldg(pred + k * a.n_t + lane), it = truth[w][lane];
+            double ape = CUDART_NAN, diff = CUDART_NAN;
+            if (ip >= 0 && ip < a.n_f && it >= 0) {
+                const double act = target_objective(a.kind[lane], __ldg(s + it), __ldg(e + it));
+                const double pre = target_objective(a.kind[lane], __ldg(s + ip), __ldg(e + ip));
+                diff = __dsub_rn(pre, act);
+                ape = __ddiv_rn(fabs(diff), fabs(act));
+            }
+            err[(k * a.n_t + lane) * 2] = ape;
+            err[(k * a.n_t + lane) * 2 + 1] = diff;
+        }
+        __syncwarp();
+    }
+}
+
+// Per-target reduction (one CTA per target, fixed order): MAPE, RMSE, count.
+__global__ void __launch_bounds__(256) k_error_reduce(const double* __restrict__ err, long long n_k, int n_t,
+                                                      double* __restrict__ summary) {
+    __shared__ double sa[256], ss[256];
+    __shared__ long long sc[256];
+    const int t = blockIdx.x;
+    double a = 0.0, q = 0.0;
+    long long c = 0;
+    for (long long k = threadIdx.x; k < n_k; k += blockDim.x) {
+        const double ape = err[(k * n_t + t) * 2], d = err[(k * n_t + t) * 2 + 1];
+        if (!isnan(ape)) { a = __dadd_rn(a, ape); q = __fma_rn(d, d, q); ++c; }
+    }
+    sa[threadIdx.x] = a; ss[threadIdx.x] = q; sc[threadIdx.x] = c;
+    __syncthreads();
+    for (int off = blockDim.x / 2; off > 0; off >>= 1) {
+        if (threadIdx.x < off) {
+            sa[threadIdx.x] += sa[threadIdx.x + off];
+            ss[threadIdx.x] += ss[threadIdx.x + off];
+            sc[threadIdx.x] += sc[threadIdx.x + off];
+        }
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        const double n = (double)sc[0];
+        summary[t * 3] = sc[0] ? sa[0] / n : CUDART_NAN;
+        summary[t * 3 + 1] = sc[0] ? sqrt(ss[0] / n) : CUDART_NAN;
+        summary[t * 3 + 2] = n;
+    }
+}
+
+// Plan emission: clock index -> MHz (HBM bound: 4 B in, 4 B out per entry).
+__global__ void __launch_bounds__(256) k_plan(const int* __restrict__ choice, long long n, const float* __restrict__ freqs,
+                                              int n_f, float* __restrict__ mhz) {
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+        const int c = __ldg(choice + i);
+        mhz[i] = (c >= 0 && c < n_f) ? __ldg(freqs + c) : CUDART_NAN_F;
+    }
+}
+
 }  // namespace syn

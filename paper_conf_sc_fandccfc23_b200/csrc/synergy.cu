@@ -296,7 +296,7 @@ bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f,
     // small batches: split each (kernel, tree) task into R clock sub-ranges so that there are at
     // least ~4 tasks per resident lane (R = 1 for large batches: every split costs an extra walk)
     const long long lanes = (long long)sm_count(0) * 1024, tasks = std::max<long long>(1, n_k * tt);
-    int nsub = (int)std::min<long long>(4, std::max<long long>(1, (4 * lanes + tasks - 1) / tasks));
+    int nsub = (int)std::min<long long>(2, std::max<long long>(1, (4 * lanes + tasks - 1) / tasks));
     nsub = std::max(1, std::min(env_int("SYNERGY_NSUB", nsub), std::max(1, n_f)));
     c.slots = nsub;                                        // carried to SweepArgs.nsub
     c.smem = da_smem(nt, kpc, n_f, c.xs, nm);
@@ -857,6 +857,75 @@ syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "k_select launch");
     g_last = {1, n_k * (long long)n_f, grid, block, 0};
+    return ok();
+}
+
+syn_status synergy_pareto(const float* d_S, const float* d_E, int64_t n_k, int32_t n_f, uint8_t* d_front,
+                          syn_stream stream) {
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    if (n_f < 1 || n_f > SYNERGY_MAX_FREQS) return fail(SYN_ERR_INVALID_ARG, "n_freqs=%d outside [1, %d]", n_f, SYNERGY_MAX_FREQS);
+    if (n_k == 0) return ok();
+    if (!d_S || !d_E || !d_front) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const long long grid = std::min<long long>((n_k + 7) / 8, (long long)sm_count(dev) * 8);
+    k_pareto<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_S, d_E, n_k, n_f, d_front);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "k_pareto launch");
+    g_last = {1, n_k * (long long)n_f, grid, 256, 0};
+    return ok();
+}
+
+syn_status synergy_choice_error(const float* d_S, const float* d_E, int64_t n_k, int32_t n_f, int32_t def,
+                                const syn_target* targets, int32_t n_t, const int32_t* d_pred, double* d_err,
+                                double* d_summary, syn_stream stream) {
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    if (n_f < 1 || n_f > SYNERGY_MAX_FREQS) return fail(SYN_ERR_INVALID_ARG, "n_freqs=%d outside [1, %d]", n_f, SYNERGY_MAX_FREQS);
+    if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
+    syn_status vs = check_targets(targets, n_t);
+    if (vs != SYN_OK) return vs;
+    if (!d_summary) return fail(SYN_ERR_INVALID_ARG, "d_summary is NULL");
+    if (n_k > 0 && (!d_S || !d_E || !d_pred || !d_err)) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    SelectArgs a;
+    memset(&a, 0, sizeof a);
+    a.S = d_S;
+    a.E = d_E;
+    a.n_k = n_k;
+    a.n_f = n_f;
+    a.def = def;
+    a.n_t = n_t;
+    for (int t = 0; t < n_t; ++t) {
+        a.kind[t] = targets[t].kind;
+        a.x[t] = targets[t].x;
+    }
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (n_k > 0) {
+        const long long grid = std::min<long long>((n_k + 7) / 8, (long long)sm_count(dev) * 8);
+        k_choice_error<<<(unsigned)grid, 256, 0, st>>>(a, d_pred, d_err);
+    }
+    k_error_reduce<<<n_t, 256, 0, st>>>(d_err, n_k, n_t, d_summary);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "k_choice_error launch");
+    g_last = {2, n_k * (long long)n_f, 0, 256, 0};
+    return ok();
+}
+
+syn_status synergy_plan(const int32_t* d_choice, int64_t n_k, int32_t n_t, const syn_clocks* clocks, float* d_mhz,
+                        syn_stream stream) {
+    if (!clocks) return fail(SYN_ERR_INVALID_ARG, "clocks is NULL");
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    if (n_t < 1 || n_t > SYNERGY_MAX_TARGETS) return fail(SYN_ERR_INVALID_ARG, "n_targets=%d outside [1, %d]", n_t, SYNERGY_MAX_TARGETS);
+    if (!current_device_is(clocks->device)) return fail(SYN_ERR_INVALID_ARG, "clocks device differs from the current device");
+    if (n_k == 0) return ok();
+    if (!d_choice || !d_mhz) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    const long long n = n_k * (long long)n_t;
+    const long long grid = std::min<long long>((n + 255) / 256, (long long)sm_count(clocks->device) * 16);
+    k_plan<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_choice, n, clocks->d_freqs, clocks->n_f, d_mhz);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "k_plan launch");
+    g_last = {1, n, grid, 256, 0};
     return ok();
 }
 

@@ -72,6 +72,9 @@ def load(path: str = LIB_PATH) -> C.CDLL:
         "synergy_select": (I32, [P, P, I64, I32, I32, P, I32, P, P]),
         "synergy_sweep": (I32, [P, P, P, I64, I32, P, I32, P, I32, P, P, P, P]),
         "synergy_sweep4": (I32, [P, P, I64, I32, P, I32, P, I32, P, P, P]),
+        "synergy_plan": (I32, [P, I64, I32, P, P, P]),
+        "synergy_pareto": (I32, [P, P, I64, I32, P, P]),
+        "synergy_choice_error": (I32, [P, P, I64, I32, I32, P, I32, P, P, P, P]),
         "synergy_workspace_create": (I32, [I32, P]),
         "synergy_workspace_destroy": (I32, [P]),
         "synergy_sweep_host": (I32, [P, P, P, P, I64, I32, P, I32, P, I32, P, P]),
@@ -253,6 +256,44 @@ def sweep4(models, features, clocks: Clocks, default_idx: int, targets, out=None
                                  _dev_ptr(out_pred, torch.float32, (4, n_k, clocks.n), "out_pred"),
                                  _stream(stream)))
     return out
+
+
+def plan(choice, clocks: Clocks, out=None, stream=None):
+    """synergy_plan: chosen clocks in MHz per kernel per target (NaN where no choice)."""
+    import torch
+    n_k, n_t = choice.shape
+    if out is None:
+        out = torch.empty((n_k, n_t), dtype=torch.float32, device=choice.device)
+    _check(load().synergy_plan(_dev_ptr(choice, torch.int32, name="choice"), n_k, n_t, clocks.handle,
+                               _dev_ptr(out, torch.float32, (n_k, n_t), "out"), _stream(stream)))
+    return out
+
+
+def pareto(S, E, out=None, stream=None):
+    """synergy_pareto: uint8 [n_k][n_f] mask of the (max S, min E) Pareto front per kernel."""
+    import torch
+    n_k, n_f = S.shape
+    if out is None:
+        out = torch.empty((n_k, n_f), dtype=torch.uint8, device=S.device)
+    _check(load().synergy_pareto(_dev_ptr(S, torch.float32, name="S"), _dev_ptr(E, torch.float32, (n_k, n_f), "E"),
+                                 n_k, n_f, _dev_ptr(out, torch.uint8, (n_k, n_f), "out"), _stream(stream)))
+    return out
+
+
+def choice_error(S_true, E_true, default_idx, targets, choice_pred, stream=None):
+    """synergy_choice_error: (err [n_k][n_t][2] = (APE, pred - actual), summary [n_t][3] =
+    (MAPE, RMSE, counted)) of predicted choices against the ground-truth table."""
+    import torch
+    n_k, n_f = S_true.shape
+    tg, n_t = _targets(targets)
+    err = torch.empty((n_k, n_t, 2), dtype=torch.float64, device=S_true.device)
+    summ = torch.empty((n_t, 3), dtype=torch.float64, device=S_true.device)
+    _check(load().synergy_choice_error(_dev_ptr(S_true, torch.float32, name="S_true"),
+                                       _dev_ptr(E_true, torch.float32, (n_k, n_f), "E_true"), n_k, n_f,
+                                       int(default_idx), tg, n_t,
+                                       _dev_ptr(choice_pred, torch.int32, (n_k, n_t), "choice_pred"),
+                                       err.data_ptr(), summ.data_ptr(), _stream(stream)))
+    return err, summ
 
 
 class Workspace:

@@ -204,6 +204,47 @@ def test_four_model_variant_lookup_tables_and_missing_models():
                 assert_bits_equal(P[m], ref["P"][m], f"model {m}")
 
 
+def test_plan_emission_mhz():
+    """NEXT f4 (L103, L187): the plan is the table clock of each choice, NaN for -1."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.make_config("c1")
+    ck = syn.Clocks(w.freqs)
+    ch = torch.from_numpy(np.array([[0, 5, -1], [w.n_freqs - 1, 7, 2]], np.int32)).cuda()
+    mhz = syn.plan(ch, ck).cpu().numpy()
+    exp = np.where(ch.cpu().numpy() >= 0, w.freqs[np.maximum(ch.cpu().numpy(), 0)], np.nan).astype(np.float32)
+    np.testing.assert_array_equal(mhz, exp)
+
+
+def test_pareto_front_and_choice_error_vs_oracle():
+    """NEXT f3 (L69, L374, L388-L392): Pareto masks bit-exact; per-kernel APE bit-exact; MAPE/RMSE
+    within 1e-12 (fixed-order GPU reduction vs sequential oracle sum)."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    rng = np.random.default_rng(21)
+    for n_f in (1, 7, 64, 196):
+        n_k = 333
+        S = (rng.integers(1, 16, (n_k, n_f)) / 8).astype(np.float32)
+        E = (rng.integers(1, 16, (n_k, n_f)) / 8).astype(np.float32)
+        S[rng.uniform(size=S.shape) < 0.03] = 0.0
+        d = int(rng.integers(0, n_f))
+        S[:, d] = 1.0
+        E[:, d] = 1.0
+        front = syn.pareto(torch.from_numpy(S).cuda(), torch.from_numpy(E).cuda()).cpu().numpy()
+        np.testing.assert_array_equal(front, oracle.pareto(S, E))
+        targets = W.targets_six() + [(W.ES, 25.0), (W.PL, 75.0)]
+        pred = rng.integers(-1, n_f, (n_k, len(targets))).astype(np.int32)
+        err, summ = syn.choice_error(torch.from_numpy(S).cuda(), torch.from_numpy(E).cuda(), d, targets,
+                                     torch.from_numpy(pred).cuda())
+        ape, mape, rmse, cnt = oracle.choice_error(S, E, d, targets, pred)
+        err = err.cpu().numpy()
+        summ = summ.cpu().numpy()
+        np.testing.assert_array_equal(err[:, :, 0], ape)
+        np.testing.assert_array_equal(summ[:, 2], cnt.astype(np.float64))
+        np.testing.assert_allclose(summ[:, 0], mape, rtol=1e-12)
+        np.testing.assert_allclose(summ[:, 1], rmse, rtol=1e-12)
+
+
 def test_empty_batch_is_noop():
     import torch
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
