@@ -419,9 +419,10 @@ def main():
                              "runs_per_kernel_tree": work["runs_per_kernel_tree"], "counted_on": work["sample"]},
                     "peak_note": f"L1/TEX load path 128 B/clk/SM x {sms} SMs x {sm_max:.0f} MHz (derived; "
                                  "not in MEASURED_PEAKS.json)",
-                    "l1_wavefront_view": {"achieved_per_s": 2.0 * blocks / kern_avg_s,
-                                          "peak_per_s": sms * sm_max * 1e6,
-                                          "note": "scattered walks: each 16-byte load is one wavefront, 2 per block"},
+                    "l1_request_view": {"achieved_per_s": blocks / kern_avg_s,
+                                        "peak_per_s": sms * sm_max * 1e6,
+                                        "note": "one 256-bit LDG (one 32-B sector, one L1 request) per block fetch; "
+                                                "peak = 1 scattered request per clk per SM"},
                     "decisions_per_s_vs_direct": evals_step * dec / kern_avg_s,
                     "hbm": hbm}
     else:
