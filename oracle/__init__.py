@@ -39,7 +39,10 @@ class _Model(C.Structure):
     _fields_ = [("n_inputs", C.c_int32), ("linear_weight", C.c_double),
                 ("lin_w", C.c_void_p), ("lin_b", C.c_double), ("forest_weight", C.c_double),
                 ("n_trees", C.c_int32), ("tree_offset", C.c_void_p), ("feature", C.c_void_p),
-                ("left", C.c_void_p), ("right", C.c_void_p), ("value", C.c_void_p)]
+                ("left", C.c_void_p), ("right", C.c_void_p), ("value", C.c_void_p),
+                ("svr_weight", C.c_double), ("n_sv", C.c_int32), ("sv", C.c_void_p), ("dual_coef", C.c_void_p),
+                ("svr_gamma", C.c_double), ("svr_intercept", C.c_double), ("in_mean", C.c_void_p),
+                ("in_scale", C.c_void_p)]
 
 
 def _load():
@@ -88,12 +91,19 @@ class _Keep:
             tree_offset=c(spec.tree_offset, dtype=np.int64), feature=c(spec.feature, dtype=np.int32),
             left=c(spec.left, dtype=np.int32), right=c(spec.right, dtype=np.int32),
             value=c(spec.value, dtype=np.float32))
+        svr = getattr(spec, "svr_weight", 0.0)
+        for k in ("sv", "dual_coef", "in_mean", "in_scale"):
+            v = getattr(spec, k, None)
+            self.arrays[k] = None if v is None else c(v, dtype=np.float32 if k == "sv" else np.float64)
         a = self.arrays
         n_trees = len(a["tree_offset"]) - 1 if spec.forest_weight != 0.0 else 0
+        n_sv = 0 if (svr == 0.0 or a["sv"] is None) else int(a["sv"].shape[0])
         self.s = _Model(int(spec.n_inputs), float(spec.linear_weight), _ptr(a["lin_w"]),
                         float(spec.lin_b), float(spec.forest_weight), int(n_trees),
                         _ptr(a["tree_offset"]), _ptr(a["feature"]), _ptr(a["left"]),
-                        _ptr(a["right"]), _ptr(a["value"]))
+                        _ptr(a["right"]), _ptr(a["value"]), float(svr), n_sv, _ptr(a["sv"]),
+                        _ptr(a["dual_coef"]), float(getattr(spec, "svr_gamma", 0.0)),
+                        float(getattr(spec, "svr_intercept", 0.0)), _ptr(a["in_mean"]), _ptr(a["in_scale"]))
 
     @property
     def ref(self):

@@ -35,6 +35,12 @@ typedef struct {
     const int32_t *left;           /* tree-local child ids                               */
     const int32_t *right;
     const float   *value;          /* threshold (internal) / leaf value                  */
+    double         svr_weight;     /* 0 => no SVR_RBF member                             */
+    int32_t        n_sv;
+    const float   *sv;             /* [n_sv][n_inputs], standardized space               */
+    const double  *dual_coef;      /* [n_sv]                                             */
+    double         svr_gamma, svr_intercept;
+    const double  *in_mean, *in_scale;  /* [n_inputs]                                    */
 } oracle_model;
 
 /* Raw model output m(x) for one input vector x[0..n_inputs-1] (fp64).

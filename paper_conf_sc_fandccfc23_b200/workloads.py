@@ -65,6 +65,19 @@ class ModelSpec:
     left: np.ndarray = field(default_factory=lambda: np.zeros(0, np.int32))
     right: np.ndarray = field(default_factory=lambda: np.zeros(0, np.int32))
     value: np.ndarray = field(default_factory=lambda: np.zeros(0, np.float32))
+    # SVR with RBF kernel (Table 2 "SVR"), scikit-learn convention on standardized
+    # inputs: svr(x) = intercept + sum_j dual_coef[j] * exp(-gamma * ||(x - in_mean)/in_scale - sv[j]||^2)
+    svr_weight: float = 0.0
+    sv: Optional[np.ndarray] = None          # float32 [n_sv][n_inputs] (standardized space)
+    dual_coef: Optional[np.ndarray] = None   # float64 [n_sv]
+    svr_gamma: float = 0.0
+    svr_intercept: float = 0.0
+    in_mean: Optional[np.ndarray] = None     # float64 [n_inputs]
+    in_scale: Optional[np.ndarray] = None    # float64 [n_inputs]
+
+    @property
+    def n_sv(self) -> int:
+        return 0 if self.svr_weight == 0.0 or self.sv is None else int(self.sv.shape[0])
 
     @property
     def n_trees(self) -> int:
@@ -82,7 +95,12 @@ class ModelSpec:
             lin_b=float(self.lin_b), forest_weight=float(self.forest_weight),
             tree_offset=c(self.tree_offset, dtype=np.int64), feature=c(self.feature, dtype=np.int32),
             left=c(self.left, dtype=np.int32), right=c(self.right, dtype=np.int32),
-            value=c(self.value, dtype=np.float32))
+            value=c(self.value, dtype=np.float32), svr_weight=float(self.svr_weight),
+            sv=None if self.sv is None else c(self.sv, dtype=np.float32),
+            dual_coef=None if self.dual_coef is None else c(self.dual_coef, dtype=np.float64),
+            svr_gamma=float(self.svr_gamma), svr_intercept=float(self.svr_intercept),
+            in_mean=None if self.in_mean is None else c(self.in_mean, dtype=np.float64),
+            in_scale=None if self.in_scale is None else c(self.in_scale, dtype=np.float64))
 
 
 @dataclass
@@ -325,6 +343,27 @@ def linear_ed2p_model(seed_seq, F, freqs, def_idx) -> ModelSpec:
     w[F] = -rng.uniform(0.3, 0.6) / f_max
     b = 1.0 - w[F] * f_def - float(np.sum(w[:F]) * 100.0)
     return ModelSpec(n_inputs=F + 1, linear_weight=1.0, lin_w=w, lin_b=b)
+
+
+def svr_energy_model(seed_seq, F, freqs, def_idx, n_sv=512, gamma=0.5) -> ModelSpec:
+    """SVR_RBF energy regressor (Table 2: SVR evaluated for MIN_ENERGY / EDP / ES), shaped like a
+    trained model: standardized inputs (log-count features, clock), support vectors drawn from the
+    input distribution, dual coefficients fitted by least squares to the analytic DVFS energy at
+    the support vectors (so predictions follow the convex energy-vs-clock shape)."""
+    rng = np.random.Generator(np.random.PCG64(seed_seq))
+    dvfs = _DVFS(rng, F, freqs, def_idx)
+    feats = np.floor(np.exp2(rng.uniform(0.0, 10.0, size=(n_sv, F))))
+    clk = freqs[rng.integers(0, len(freqs), size=n_sv)].astype(np.float64)
+    X = np.concatenate([feats, clk[:, None]], axis=1)
+    mean = np.concatenate([np.full(F, 256.0), [float(np.mean(freqs))]])
+    scale = np.concatenate([np.full(F, 300.0), [float(np.std(freqs))]])
+    Z = ((X - mean) / scale).astype(np.float32)
+    y = dvfs.energy(dvfs.beta(feats), clk)
+    K = np.exp(-gamma * ((Z[:, None, :].astype(np.float64) - Z[None, :, :]) ** 2).sum(-1))
+    b = float(np.mean(y))
+    dual = np.linalg.solve(K + 1e-2 * np.eye(n_sv), y - b)
+    return ModelSpec(n_inputs=F + 1, svr_weight=1.0, sv=Z, dual_coef=dual, svr_gamma=gamma,
+                     svr_intercept=b, in_mean=mean, in_scale=scale)
 
 
 # ------------------------------------------------------------------------ configs

@@ -168,3 +168,48 @@ def test_sklearn_forest_full_pipeline_normalised(oracle_lib):
         Xi = np.concatenate([feats, np.full((20, 1), f, np.float32)], axis=1)
         P[:, i] = rf.predict(Xi)
     np.testing.assert_array_equal(S, (P / P[:, d:d + 1]).astype(np.float32))
+
+
+def export_svr(pipe, n_inputs):
+    """sklearn Pipeline(StandardScaler, SVR(kernel="rbf")) -> ModelSpec SVR member; the support
+    vectors are rounded to fp32 (the model format) and written back into the sklearn SVR."""
+    scaler, svr = pipe.named_steps["standardscaler"], pipe.named_steps["svr"]
+    sv32 = svr.support_vectors_.astype(np.float32)
+    svr.support_vectors_[:] = sv32.astype(np.float64)
+    svr._sparse = False
+    return W.ModelSpec(n_inputs=n_inputs, svr_weight=1.0, sv=sv32, dual_coef=svr.dual_coef_[0].copy(),
+                       svr_gamma=float(svr._gamma), svr_intercept=float(svr.intercept_[0]),
+                       in_mean=scaler.mean_.copy(), in_scale=scaler.scale_.copy())
+
+
+def test_svr_rbf_matches_sklearn(oracle_lib):
+    """SVR with RBF kernel (Table 2) on standardized inputs: scikit-learn predictions."""
+    from sklearn.pipeline import make_pipeline
+    from sklearn.preprocessing import StandardScaler
+    from sklearn.svm import SVR
+    rng = np.random.default_rng(12)
+    F = 5
+    X, y = _dvfs_data(rng, 600, F, W.clock_table(64))
+    pipe = make_pipeline(StandardScaler(), SVR(kernel="rbf", gamma=0.3, C=3.0, epsilon=0.01)).fit(X.astype(np.float64), y)
+    spec = export_svr(pipe, F + 1)
+    assert spec.n_sv > 50
+    Xt = X[:200]
+    ref = pipe.predict(Xt.astype(np.float64))
+    got = np.array([oracle_lib.model_eval(spec, x) for x in Xt])
+    np.testing.assert_allclose(got, ref, rtol=1e-11, atol=1e-12)
+
+
+def test_svr_closed_form_and_ensemble_order(oracle_lib):
+    """Two support vectors in 2-D with hand-computed distances; svr joins the ensemble last (Q7)."""
+    spec = W.ModelSpec(n_inputs=2, svr_weight=1.0, sv=np.array([[0.0, 0.0], [1.0, -1.0]], np.float32),
+                       dual_coef=np.array([2.0, -0.5]), svr_gamma=0.25, svr_intercept=0.125,
+                       in_mean=np.array([1.0, 10.0]), in_scale=np.array([2.0, 4.0]))
+    x = np.array([3.0, 6.0], np.float32)        # z = (1, -1): d0^2 = 2, d1^2 = 0
+    assert abs(oracle_lib.model_eval(spec, x) - (0.125 + 2.0 * np.exp(-0.5) - 0.5)) < 1e-15
+    x = np.array([1.0, 10.0], np.float32)       # z = (0, 0): d0^2 = 0, d1^2 = 2
+    assert abs(oracle_lib.model_eval(spec, x) - (0.125 + 2.0 - 0.5 * np.exp(-0.5))) < 1e-15
+    both = W.ModelSpec(n_inputs=2, svr_weight=0.5, sv=spec.sv, dual_coef=spec.dual_coef, svr_gamma=0.25,
+                       svr_intercept=0.125, in_mean=spec.in_mean, in_scale=spec.in_scale,
+                       linear_weight=2.0, lin_w=np.array([1.0, 0.0]), lin_b=0.0)
+    want = 2.0 * 1.0 + 0.5 * (0.125 + 2.0 - 0.5 * np.exp(-0.5))
+    assert abs(oracle_lib.model_eval(both, x) - want) < 1e-15
