@@ -24,7 +24,8 @@
  *     stream).  Results are valid after the caller synchronises that stream.  Launch failures
  *     return SYN_ERR_CUDA.
  *   - "d_" pointers are device pointers on the model's device, "h_" pointers host pointers.
- *     The caller owns every buffer it passes; the hot calls never allocate.
+ *     The caller owns every buffer it passes; the hot calls never allocate, except the
+ *     stream-ordered SVR scratch described at syn_model_desc.
  *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
  *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
  *   - Handles (models, clock tables, workspaces) are bound to the device they were created
@@ -40,7 +41,7 @@
 extern "C" {
 #endif
 
-#define SYNERGY_VERSION 1
+#define SYNERGY_VERSION 2
 #define SYNERGY_MAX_FREQS 4096
 #define SYNERGY_MAX_TARGETS 16
 #define SYNERGY_MAX_INPUTS 255
@@ -78,9 +79,21 @@ typedef void *syn_stream;   /* cudaStream_t */
  * in MHz; inputs 0..n_inputs-2 are the static features.  Output (Q7/Q8):
  *   m(x) = 0;  m += linear_weight * (lin_b + sum_j lin_w[j] x[j])   if linear_weight != 0
  *              m += forest_weight * mean_t leaf_t(x)                if forest_weight != 0
+ *              m += svr_weight * svr(x)                             if svr_weight != 0
  * in fp64: fp64 fma over j in order for the linear member; for the forest the exact sum of the
  * fp32 leaves rounded once to fp64 (order-free, Q8), then / n_trees; a weight of
- * exactly 1 skips its multiplication. */
+ * exactly 1 skips its multiplication.
+ * SVR with RBF kernel (Table 2 "SVR"; scikit-learn SVR on StandardScaler inputs):
+ *   svr(x) = svr_intercept + sum_j dual_coef[j] * exp(-svr_gamma * ||z(x) - sv[j]||^2),
+ *   z(x)_d = (x[d] - in_mean[d]) / in_scale[d],
+ * fp64.  Over a clock sweep the squared distance splits into a static-feature part and a
+ * clock part, so the device evaluates sum_j (dual_j e^{-gamma A_kj}) e^{-gamma B_ji}: a
+ * [kernels x SVs] x [SVs x clocks] fp64 contraction (Q24).  It agrees with the plain
+ * definition within 2^-40 * (|svr_intercept| + sum_j |dual_coef[j]|), NOT bit for bit.
+ * Calls whose models have an SVR member take scratch of (n_sv + splits * n_kernels) * n_freqs
+ * * 8 bytes per SVR model from the device's default stream-ordered memory pool
+ * (cudaMallocAsync / cudaFreeAsync on the call's stream; splits <= 16), the only allocation a
+ * hot call makes. */
 typedef struct {
     int32_t n_inputs;            /* F + 1, 1 .. SYNERGY_MAX_INPUTS                        */
     double linear_weight;        /* 0 => no linear member                                 */
@@ -93,6 +106,14 @@ typedef struct {
     const int32_t *left;         /* [n_nodes] tree-local child ids (ignored at leaves)    */
     const int32_t *right;
     const float *value;          /* [n_nodes] threshold or leaf value                     */
+    double svr_weight;           /* 0 => no SVR_RBF member (the fields below are ignored) */
+    int32_t n_sv;                /* support vectors, 1 .. 2^24                            */
+    const float *sv;             /* [n_sv][n_inputs] support vectors, standardized space  */
+    const double *dual_coef;     /* [n_sv] dual coefficients (alpha_j - alpha_j^*)        */
+    double svr_gamma;            /* RBF gamma, finite, >= 0                               */
+    double svr_intercept;
+    const double *in_mean;       /* [n_inputs] standardization, in_scale finite and != 0  */
+    const double *in_scale;
 } syn_model_desc;
 
 typedef struct syn_model syn_model;      /* opaque, device-resident, immutable */
@@ -105,7 +126,8 @@ int32_t synergy_version(void);
 
 /* Validate, re-lay (breadth-first, children adjacent) and upload a model to `device`.
  * INVALID_ARG: null arrays, n_inputs out of range, a child id outside its tree, a node
- * reached twice (not a tree), a split feature outside [0, n_inputs), both weights 0.
+ * reached twice (not a tree), a split feature outside [0, n_inputs), all member weights 0,
+ * an SVR member with NULL arrays, n_sv outside [1, 2^24], non-finite values or a zero scale.
  * UNSUPPORTED: depth > SYNERGY_MAX_DEPTH or more than 2^31-2 nodes.  OOM / CUDA otherwise.
  * Synchronous (returns after the upload). */
 syn_status synergy_model_create(const syn_model_desc *desc, int32_t device, syn_model **out);

@@ -42,6 +42,41 @@ struct DevModel {
     int fx_ok;
     double fx_scale;         // 2^s
     double fx_inv;           // 2^-s
+    // SVR_RBF member: svr = b + sum_j dual_j exp(-gamma ||(x - mean)/scale - sv_j||^2)
+    double svr_weight;       // 0 => absent
+    int n_sv;
+    const float* sv;         // [n_sv][n_inputs]
+    const double* dual;      // [n_sv]
+    const double* in_mean;   // [n_inputs]
+    const double* in_scale;  // [n_inputs]
+    double svr_gamma, svr_b;
+    // per call (k_svr): svr_splits partial contractions over SV ranges, [svr_splits][n_k][n_f],
+    // summed in split order (+ svr_b) by finish_tile
+    const double* svr_p;
+    int svr_splits;
+};
+
+// k_svr tiling: 8 warps x kSvrRows kernels per CTA, 32 x CPT clocks, SVs staged kSvrJC at a time
+constexpr int kSvrRows = 8;
+constexpr int kSvrTK = 8 * kSvrRows;
+constexpr int kSvrJC = 16;
+constexpr int kSvrMaxSplits = 16;
+
+struct SvrArgs {
+    const float* features;   // [n_k][F]
+    long long n_k;
+    int F;
+    const float* freqs;      // [n_f]
+    int n_f;
+    const float* sv;
+    const double* dual;
+    const double* in_mean;
+    const double* in_scale;
+    double gamma;
+    int n_sv;
+    int sv_per_split;        // SV range of split blockIdx.z
+    double* V;               // [n_sv][n_f] clock factors e^{-gamma B_ji}
+    double* P;               // [splits][n_k][n_f]
 };
 
 constexpr int kMaxTargets = 16;

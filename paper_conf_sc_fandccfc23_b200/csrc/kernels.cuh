@@ -16,6 +16,7 @@
 #include <cstdint>
 
 #include "internal.h"
+#include "kernels_svr.cuh"
 
 namespace syn {
 
@@ -164,17 +165,19 @@ __device__ __forceinline__ void select_row_warp(const float* S, const float* E, 
 // clock (S = (float)(mS_i / mS_def), L69 / DESIGN.md Q13; raw (float)m when def == -1), write
 // the predictions if requested, then run the per-target selection.  mS/mE: [nk][n_f] doubles,
 // sS/sE: [nk][n_f] float scratch, all in shared memory.  Caller has synchronised the block.
-__device__ __forceinline__ void finish_tile(const SweepArgs& a, const double* mS, const double* mE,
+__device__ __forceinline__ void finish_tile(const SweepArgs& a, double* mS, double* mE,
                                             float* sS, float* sE, int nk, long long k0) {
     const int n_f = a.n_f;
     const int lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;
     for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
-        const double* rS = mS + (size_t)kl * n_f;
-        const double* rE = mE + (size_t)kl * n_f;
+        double* rS = mS + (size_t)kl * n_f;
+        double* rE = mE + (size_t)kl * n_f;
         float* oS = sS + (size_t)kl * n_f;
         float* oE = sE + (size_t)kl * n_f;
         const long long k = k0 + kl;
+        add_svr_row(a.ms, rS, k, a.n_k, n_f, lane);       // SVR member last (ensemble order, Q7)
+        add_svr_row(a.me, rE, k, a.n_k, n_f, lane);
         const double dS = a.def >= 0 ? rS[a.def] : 1.0;
         const double dE = a.def >= 0 ? rE[a.def] : 1.0;
         for (int i = lane; i < n_f; i += 32) {
@@ -202,7 +205,8 @@ __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* 
         const long long k = k0 + kl;
         for (int m = 0; m < 4; ++m) {
             if (!mv[m]) continue;
-            const double* r = mv[m] + (size_t)kl * n_f;
+            double* r = mv[m] + (size_t)kl * n_f;
+            add_svr_row(m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2], r, k, a.n_k, n_f, lane);
             float* o = sv[m] + (size_t)kl * n_f;
             float* g = m == 0 ? a.S_out : m == 1 ? a.E_out : a.X_out[m - 2];
             const double dv = a.def >= 0 ? r[a.def] : 1.0;

@@ -17,6 +17,7 @@
 #include "kernels_iv.cuh"
 #include "kernels_ws.cuh"
 #include "kernels_da.cuh"
+#include "kernels_svr.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -365,6 +366,98 @@ syn_status validate_sweep(const syn_model* sp, const syn_model* en, int64_t n_k,
     return SYN_OK;
 }
 
+// SVR members (kernels_svr.cuh): per model, V = clock factors and the split contractions P into
+// stream-ordered scratch; dm.svr_p / svr_splits point the finish step at them.  Released with
+// release() after the sweep kernel is enqueued (cudaFreeAsync keeps it alive until then).
+struct SvrScratch {
+    std::vector<void*> bufs;
+    cudaStream_t st = nullptr;
+    int launches = 0;
+    void release() {
+        for (void* b : bufs) cudaFreeAsync(b, st);
+        bufs.clear();
+    }
+    ~SvrScratch() { release(); }
+};
+
+template <int CPT>
+cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, size_t smem, cudaStream_t st) {
+    static size_t smem_set = 48 * 1024;
+    if (smem > smem_set) {
+        cudaError_t e = cudaFuncSetAttribute(k_svr<CPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        smem_set = smem;
+    }
+    k_svr<CPT><<<grid, 256, smem, st>>>(sa);
+    return cudaGetLastError();
+}
+
+syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
+                       cudaStream_t st, SvrScratch& scr) {
+    if (dm.svr_weight == 0.0) return ok();
+    scr.st = st;
+    const int n_f = clocks->n_f;
+    const int cpt = std::min(8, (n_f + 31) / 32);
+    const int tn = 32 * cpt;
+    const long long tiles_n = (n_f + tn - 1) / tn;
+    const long long tiles = (n_k + kSvrTK - 1) / kSvrTK * tiles_n;
+    if ((n_k + kSvrTK - 1) / kSvrTK > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for k_svr");
+    // split the SV range across CTAs until the grid covers the SMs (at most kSvrMaxSplits)
+    long long splits = std::max<long long>(1, sm_count(device) / std::max<long long>(tiles, 1));
+    splits = std::min<long long>(splits, kSvrMaxSplits);
+    splits = env_int("SYNERGY_SVR_SPLITS", (int)splits);
+    splits = std::max<long long>(1, std::min<long long>(splits, (dm.n_sv + kSvrJC - 1) / kSvrJC));
+    const int per = (int)(((dm.n_sv + splits - 1) / splits + kSvrJC - 1) / kSvrJC * kSvrJC);
+    splits = (dm.n_sv + per - 1) / per;
+    const size_t vb = (size_t)dm.n_sv * n_f * sizeof(double);
+    const size_t pb = (size_t)splits * (size_t)n_k * n_f * sizeof(double);
+    const size_t voff = (pb + 255) / 256 * 256;
+    void* buf = nullptr;
+    cudaError_t e = cudaMallocAsync(&buf, voff + vb, st);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "SVR scratch of %zu bytes", voff + vb)
+                                              : cuda_fail(e, "cudaMallocAsync(SVR scratch)");
+    }
+    scr.bufs.push_back(buf);
+    SvrArgs sa;
+    memset(&sa, 0, sizeof sa);
+    sa.features = d_features;
+    sa.n_k = n_k;
+    sa.F = F;
+    sa.freqs = clocks->d_freqs;
+    sa.n_f = n_f;
+    sa.sv = dm.sv;
+    sa.dual = dm.dual;
+    sa.in_mean = dm.in_mean;
+    sa.in_scale = dm.in_scale;
+    sa.gamma = dm.svr_gamma;
+    sa.n_sv = dm.n_sv;
+    sa.sv_per_split = per;
+    sa.P = static_cast<double*>(buf);
+    sa.V = reinterpret_cast<double*>(static_cast<char*>(buf) + voff);
+    const long long nv = (long long)dm.n_sv * n_f;
+    k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
+    if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "k_svr_v launch");
+    const size_t smem = ((size_t)F * kSvrTK + (size_t)kSvrJC * kSvrTK + (size_t)kSvrJC * tn) * sizeof(double);
+    const dim3 grid((unsigned)((n_k + kSvrTK - 1) / kSvrTK), (unsigned)tiles_n, (unsigned)splits);
+    switch (cpt) {
+        case 1: e = launch_svr_t<1>(sa, grid, smem, st); break;
+        case 2: e = launch_svr_t<2>(sa, grid, smem, st); break;
+        case 3: e = launch_svr_t<3>(sa, grid, smem, st); break;
+        case 4: e = launch_svr_t<4>(sa, grid, smem, st); break;
+        case 5: e = launch_svr_t<5>(sa, grid, smem, st); break;
+        case 6: e = launch_svr_t<6>(sa, grid, smem, st); break;
+        case 7: e = launch_svr_t<7>(sa, grid, smem, st); break;
+        default: e = launch_svr_t<8>(sa, grid, smem, st); break;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "k_svr launch");
+    scr.launches += 2;
+    dm.svr_p = sa.P;
+    dm.svr_splits = (int)splits;
+    return ok();
+}
+
 syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
                      int32_t F, const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
                      int32_t* d_choice, float* d_S, float* d_E, int mode, cudaStream_t st) {
@@ -432,13 +525,17 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     a.nsub = c.algo == 3 ? c.slots : 1;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
+    SvrScratch scr;
+    syn_status ss = prepare_svr(a.ms, clocks->device, d_features, n_k, F, clocks, st, scr);
+    if (ss == SYN_OK) ss = prepare_svr(a.me, clocks->device, d_features, n_k, F, clocks, st, scr);
+    if (ss != SYN_OK) return ss;
     cudaError_t e = c.algo == 3 ? launch_da(a, c, grid, st)
                   : c.algo == 2 ? launch_ws(a, c, grid, st)
                   : c.algo == 1 ? launch_iv(a, c, grid, st)
                                 : launch_sweep(a, c, grid, st);
     static const char* names[4] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch", "k_sweep_da launch"};
     if (e != cudaSuccess) return cuda_fail(e, names[c.algo]);
-    g_last = {1, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
+    g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
     return ok();
 }
 
@@ -458,12 +555,27 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     if (!d) return fail(SYN_ERR_INVALID_ARG, "desc is NULL");
     if (d->n_inputs < 1 || d->n_inputs > SYNERGY_MAX_INPUTS)
         return fail(SYN_ERR_INVALID_ARG, "n_inputs=%d outside [1, %d]", d->n_inputs, SYNERGY_MAX_INPUTS);
-    if (!std::isfinite(d->linear_weight) || !std::isfinite(d->forest_weight))
+    if (!std::isfinite(d->linear_weight) || !std::isfinite(d->forest_weight) || !std::isfinite(d->svr_weight))
         return fail(SYN_ERR_INVALID_ARG, "member weights must be finite");
-    if (d->linear_weight == 0.0 && d->forest_weight == 0.0)
-        return fail(SYN_ERR_INVALID_ARG, "both member weights are 0");
+    if (d->linear_weight == 0.0 && d->forest_weight == 0.0 && d->svr_weight == 0.0)
+        return fail(SYN_ERR_INVALID_ARG, "all member weights are 0");
     if (d->linear_weight != 0.0 && !d->lin_w) return fail(SYN_ERR_INVALID_ARG, "lin_w is NULL");
     const int F = d->n_inputs - 1;
+    const bool has_svr = d->svr_weight != 0.0;
+    if (has_svr) {
+        if (d->n_sv < 1 || d->n_sv > (1 << 24)) return fail(SYN_ERR_INVALID_ARG, "n_sv=%d outside [1, 2^24]", d->n_sv);
+        if (!d->sv || !d->dual_coef || !d->in_mean || !d->in_scale)
+            return fail(SYN_ERR_INVALID_ARG, "SVR arrays must be non-NULL");
+        if (!std::isfinite(d->svr_gamma) || d->svr_gamma < 0.0 || !std::isfinite(d->svr_intercept))
+            return fail(SYN_ERR_INVALID_ARG, "svr_gamma must be finite and >= 0, svr_intercept finite");
+        for (int64_t q = 0; q < (int64_t)d->n_sv * d->n_inputs; ++q)
+            if (!std::isfinite(d->sv[q])) return fail(SYN_ERR_INVALID_ARG, "sv[%lld] is not finite", (long long)q);
+        for (int j = 0; j < d->n_sv; ++j)
+            if (!std::isfinite(d->dual_coef[j])) return fail(SYN_ERR_INVALID_ARG, "dual_coef[%d] is not finite", j);
+        for (int q = 0; q < d->n_inputs; ++q)
+            if (!std::isfinite(d->in_mean[q]) || !std::isfinite(d->in_scale[q]) || d->in_scale[q] == 0.0)
+                return fail(SYN_ERR_INVALID_ARG, "in_mean/in_scale[%d] not finite or scale 0", q);
+    }
     const uint32_t leaf_code = (uint32_t)(F + 1);
     std::vector<uint2> nodes;
     std::vector<int2> trees;
@@ -615,7 +727,11 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     const size_t rb = std::max<size_t>(broot.size(), 1) * sizeof(int);
     const size_t off_t = (nb + 255) / 256 * 256, off_l = off_t + (tb + 255) / 256 * 256;
     const size_t off_b = off_l + (lb + 255) / 256 * 256, off_r = off_b + (bb + 255) / 256 * 256;
-    const size_t total = off_r + rb;
+    const size_t n_sv = has_svr ? (size_t)d->n_sv : 0;
+    const size_t svb = n_sv * d->n_inputs * sizeof(float), dcb = n_sv * sizeof(double);
+    const size_t off_sv = off_r + (rb + 255) / 256 * 256, off_dc = off_sv + (svb + 255) / 256 * 256;
+    const size_t off_mn = off_dc + (dcb + 255) / 256 * 256, off_sc = off_mn + (lb + 255) / 256 * 256;
+    const size_t total = has_svr ? off_sc + lb : off_r + rb;
     void* mem = nullptr;
     cudaError_t e = cudaMalloc(&mem, total);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(model)");
@@ -626,7 +742,11 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         (!trees.empty() && (e = cudaMemcpy(base + off_t, trees.data(), trees.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
         (!blocks.empty() && (e = cudaMemcpy(base + off_b, blocks.data(), blocks.size() * sizeof(uint4), cudaMemcpyHostToDevice)) != cudaSuccess) ||
-        (!broot.empty() && (e = cudaMemcpy(base + off_r, broot.data(), broot.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess)) {
+        (!broot.empty() && (e = cudaMemcpy(base + off_r, broot.data(), broot.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess) ||
+        (has_svr && ((e = cudaMemcpy(base + off_sv, d->sv, svb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+                     (e = cudaMemcpy(base + off_dc, d->dual_coef, dcb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+                     (e = cudaMemcpy(base + off_mn, d->in_mean, lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+                     (e = cudaMemcpy(base + off_sc, d->in_scale, lb, cudaMemcpyHostToDevice)) != cudaSuccess))) {
         cudaFree(mem);
         return cuda_fail(e, "cudaMemcpy(model)");
     }
@@ -635,6 +755,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         cudaFree(mem);
         return fail(SYN_ERR_OOM, "host allocation failed");
     }
+    memset(&m->dm, 0, sizeof m->dm);
     m->device = device;
     m->n_inputs = d->n_inputs;
     m->n_trees = d->forest_weight != 0.0 ? d->n_trees : 0;
@@ -657,6 +778,18 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.fx_ok = fx_ok;
     m->dm.fx_scale = std::ldexp(1.0, fx_s);
     m->dm.fx_inv = std::ldexp(1.0, -fx_s);
+    m->dm.svr_weight = d->svr_weight;
+    m->dm.n_sv = (int)n_sv;
+    if (has_svr) {
+        m->dm.sv = reinterpret_cast<const float*>(base + off_sv);
+        m->dm.dual = reinterpret_cast<const double*>(base + off_dc);
+        m->dm.in_mean = reinterpret_cast<const double*>(base + off_mn);
+        m->dm.in_scale = reinterpret_cast<const double*>(base + off_sc);
+        m->dm.svr_gamma = d->svr_gamma;
+        m->dm.svr_b = d->svr_intercept;
+    }
+    m->dm.svr_p = nullptr;
+    m->dm.svr_splits = 0;
     *out = m;
     return ok();
 }
@@ -817,9 +950,16 @@ syn_status synergy_sweep4(const syn_model* const* models, const float* d_feature
     a.nsub = c.slots;
     const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
     if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    cudaError_t e = launch_da(a, c, grid, static_cast<cudaStream_t>(stream));
+    const cudaStream_t st = static_cast<cudaStream_t>(stream);
+    SvrScratch scr;
+    syn_status ss = SYN_OK;
+    DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
+    for (int m = 0; m < 4 && ss == SYN_OK; ++m)
+        if (m < 2 || a.has_x[m - 2]) ss = prepare_svr(*dms[m], clocks->device, d_features, n_k, F, clocks, st, scr);
+    if (ss != SYN_OK) return ss;
+    cudaError_t e = launch_da(a, c, grid, st);
     if (e != cudaSuccess) return cuda_fail(e, "k_sweep_da launch");
-    g_last = {1, n_k * (long long)n_f, grid, c.nt, 3000 + c.tile_k};
+    g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, 3000 + c.tile_k};
     return ok();
 }
 

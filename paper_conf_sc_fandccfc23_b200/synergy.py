@@ -38,7 +38,9 @@ class _ModelDesc(C.Structure):
     _fields_ = [("n_inputs", C.c_int32), ("linear_weight", C.c_double), ("lin_w", C.c_void_p),
                 ("lin_b", C.c_double), ("forest_weight", C.c_double), ("n_trees", C.c_int32),
                 ("tree_offset", C.c_void_p), ("feature", C.c_void_p), ("left", C.c_void_p),
-                ("right", C.c_void_p), ("value", C.c_void_p)]
+                ("right", C.c_void_p), ("value", C.c_void_p), ("svr_weight", C.c_double),
+                ("n_sv", C.c_int32), ("sv", C.c_void_p), ("dual_coef", C.c_void_p), ("svr_gamma", C.c_double),
+                ("svr_intercept", C.c_double), ("in_mean", C.c_void_p), ("in_scale", C.c_void_p)]
 
 
 _lib = None
@@ -136,6 +138,17 @@ class Model:
         d = _ModelDesc(int(spec.n_inputs), float(spec.linear_weight), None if lw is None else lw.ctypes.data,
                        float(spec.lin_b), float(spec.forest_weight), int(n_trees), off.ctypes.data,
                        fe.ctypes.data, le.ctypes.data, ri.ctypes.data, va.ctypes.data)
+        svr_w = float(getattr(spec, "svr_weight", 0.0))
+        if svr_w != 0.0:
+            sv = c(spec.sv, dtype=np.float32)
+            du, mn, sc = (c(spec.dual_coef, dtype=np.float64), c(spec.in_mean, dtype=np.float64),
+                          c(spec.in_scale, dtype=np.float64))
+            self._keep += [sv, du, mn, sc]
+            d.svr_weight = svr_w
+            d.n_sv = int(sv.shape[0])
+            d.sv, d.dual_coef, d.in_mean, d.in_scale = sv.ctypes.data, du.ctypes.data, mn.ctypes.data, sc.ctypes.data
+            d.svr_gamma = float(spec.svr_gamma)
+            d.svr_intercept = float(spec.svr_intercept)
         h = C.c_void_p()
         _check(lib.synergy_model_create(C.byref(d), int(device), C.byref(h)))
         self._h = h

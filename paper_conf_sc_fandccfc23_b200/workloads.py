@@ -418,6 +418,21 @@ def make_models4(cfg: str = "c2"):
              linear_ed2p_model(s_ed2p, N_STATIC, freqs, d)], freqs, d)
 
 
+def make_models_svr(cfg: str = "c2", n_sv: int = 512, ensemble: bool = False):
+    """SVR variant (Table 2 "SVR") on config cfg's shapes: the
+    config's speedup model and an SVR_RBF energy model (n_sv support vectors).  ensemble=True
+    instead makes the energy model 0.5 * forest + 0.5 * SVR (the weighted-ensemble reading Q7)."""
+    sp, en, freqs, d = make_models(cfg)
+    ss = np.random.SeedSequence(SEED_BASE + 200 + CONFIG_INDEX[cfg])
+    svr = svr_energy_model(ss, N_STATIC, freqs, d, n_sv=n_sv)
+    if ensemble:
+        svr = ModelSpec(n_inputs=en.n_inputs, forest_weight=0.5, tree_offset=en.tree_offset, feature=en.feature,
+                        left=en.left, right=en.right, value=en.value, svr_weight=0.5, sv=svr.sv,
+                        dual_coef=svr.dual_coef, svr_gamma=svr.svr_gamma, svr_intercept=svr.svr_intercept,
+                        in_mean=svr.in_mean, in_scale=svr.in_scale)
+    return sp, svr, freqs, d
+
+
 def make_features(cfg: str, row0: int = 0, n: Optional[int] = None) -> np.ndarray:
     n_k = CONFIGS[cfg][0]
     feat_ss, _, _ = _seeds(cfg)

@@ -37,7 +37,7 @@ def test_library_is_sm100a(lib):
 
 
 def test_version_and_error_string(lib):
-    assert lib.synergy_version() == 1
+    assert lib.synergy_version() == 2
     h = C.c_void_p()
     assert lib.synergy_model_create(None, 0, C.byref(h)) == syn.SYN_ERR_INVALID_ARG
     assert b"desc" in lib.synergy_last_error()
@@ -82,3 +82,41 @@ def test_model_validation(lib):
     assert create(badf) == syn.SYN_ERR_INVALID_ARG                         # feature >= n_inputs
     none = W.ModelSpec(n_inputs=3)
     assert create(none) == syn.SYN_ERR_INVALID_ARG                         # no member
+
+
+def test_model_desc_layout_matches_header():
+    """The binding's ctypes struct lists syn_model_desc's fields in header order."""
+    import re
+    src = open(syn.HEADER).read()
+    body = src[src.index("typedef struct {\n    int32_t n_inputs;"):src.index("} syn_model_desc;")]
+    names = re.findall(r"\b(\w+);", body)
+    assert [f for f, _ in syn._ModelDesc._fields_] == names
+
+
+@pytest.mark.parametrize("bad", ["scale0", "nsv0", "nan_dual", "neg_gamma", "null_sv", "nan_sv"])
+def test_svr_model_validation(lib, bad):
+    """SVR members are validated on the host (synergy.h: synergy_model_create)."""
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    _, en, _, _ = W.make_models_svr("c1", n_sv=20)
+    en.in_scale = en.in_scale.copy()
+    en.dual_coef = en.dual_coef.copy()
+    en.sv = en.sv.copy()
+    if bad == "scale0":
+        en.in_scale[2] = 0.0
+    elif bad == "nsv0":
+        en.sv = en.sv[:0]
+    elif bad == "nan_dual":
+        en.dual_coef[3] = np.nan
+    elif bad == "neg_gamma":
+        en.svr_gamma = -1.0
+    elif bad == "nan_sv":
+        en.sv[5, 1] = np.inf
+    with pytest.raises(syn.SynergyError) as ei:
+        if bad == "null_sv":
+            d = syn._ModelDesc(en.n_inputs, 0.0, None, 0.0, 0.0, 0, None, None, None, None, None, 1.0, 4, None,
+                               None, 0.5, 0.0, None, None)
+            h = C.c_void_p()
+            syn._check(lib.synergy_model_create(C.byref(d), 0, C.byref(h)))
+        else:
+            syn.Model(en)
+    assert ei.value.status == syn.SYN_ERR_INVALID_ARG
