@@ -41,6 +41,9 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--flush-mib", type=int, default=512)
+    p.add_argument("--models", default="rf", choices=["rf", "svr"],
+                   help="rf: the config's models (north star); svr: the config's speedup model + an "
+                        "SVR_RBF energy model with 512 support vectors (SURVEY NEXT f2)")
     return p.parse_args()
 
 
@@ -49,13 +52,23 @@ def dist_env():
             int(os.environ.get("LOCAL_RANK", 0)))
 
 
-def workload_desc(cfg):
+def bench_models(cfg, which="rf"):
+    """(speedup, energy, freqs, default_idx) of the benchmarked workload."""
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    return W.make_models(cfg) if which == "rf" else W.make_models_svr(cfg, n_sv=SVR_SV)
+
+
+SVR_SV = 512
+
+
+def workload_desc(cfg, which="rf"):
     from paper_conf_sc_fandccfc23_b200 import workloads as W
     n_k, n_f, sp, en, tg = W.CONFIGS[cfg]
     m = lambda s: "linear" if s[0] == "lin" else f"RF {s[1]}xD{s[2]}"
     tgt = "MAX_PERF,MIN_ENERGY,MIN_EDP,MIN_ED2P,ES_50,PL_50" if tg == "six" else "ES_25,ES_50,ES_75,PL_25,PL_50,PL_75"
-    return (f"{cfg}: {n_k} kernels x {n_f} core clocks, speedup {m(sp)}, energy {m(en)}, 12 static "
-            f"features, targets {tgt}")
+    ens = m(en) if which == "rf" else f"SVR_RBF {SVR_SV} SVs"
+    return (f"{cfg}{'' if which == 'rf' else '+svr'}: {n_k} kernels x {n_f} core clocks, speedup {m(sp)}, "
+            f"energy {ens}, 12 static features, targets {tgt}")
 
 
 def decisions_per_eval(spec):
@@ -162,21 +175,21 @@ def _oracle_range(args):
 _POOL_CACHE = {}
 
 
-def _pool_init(cfg):
+def _pool_init(cfg, which="rf"):
     from paper_conf_sc_fandccfc23_b200 import workloads as W
     import oracle
     oracle.build()
-    sp, en, freqs, d = W.make_models(cfg)
+    sp, en, freqs, d = bench_models(cfg, which)
     tg = W.targets_six() if W.CONFIGS[cfg][4] == "six" else W.targets_es_pl()
     _POOL_CACHE[cfg] = (sp, en, freqs, d, tg)
 
 
-def oracle_single_core(cfg, n_k_cap, budget_s=10.0):
+def oracle_single_core(cfg, n_k_cap, budget_s=10.0, which="rf"):
     """The oracle as it stands, one core, on the first kernels of the workload until ~budget_s."""
     import oracle
     from paper_conf_sc_fandccfc23_b200 import workloads as W
     oracle.build()
-    w = W.make_config(cfg, row0=0, n=min(n_k_cap, W.CONFIGS[cfg][0]))
+    w = W.make_config(cfg, row0=0, n=min(n_k_cap, W.CONFIGS[cfg][0]), models=bench_models(cfg, which))
     evals = 0
     t0 = time.perf_counter()
     chunk = max(1, min(w.n_kernels, 100))
@@ -195,19 +208,20 @@ def oracle_single_core(cfg, n_k_cap, budget_s=10.0):
     return evals / el, evals, el
 
 
-def run_walk_work(cfg, row0, n_rows, budget=5e8):
+def run_walk_work(cfg, row0, n_rows, budget=5e8, which="rf"):
     """Run-walk work of the launched rows, counted by the oracle on the first rows that fit a
     budget of ~5e8 node decisions (all rows for c1/c2/c5): runs of clocks sharing a leaf and their
     2-level block fetches."""
     import oracle
     from paper_conf_sc_fandccfc23_b200 import workloads as W
     n_f = W.CONFIGS[cfg][1]
-    sp, en = W.make_models(cfg)[:2]
+    models = bench_models(cfg, which)
+    sp, en = models[:2]
     per_row = max(1, n_f * (decisions_per_eval(sp) + decisions_per_eval(en)))
     n = int(min(n_rows, max(16, budget // per_row)))
     if n == 0:
         return None
-    w = W.make_config(cfg, row0=row0, n=n)
+    w = W.make_config(cfg, row0=row0, n=n, models=models)
     r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
     trees = w.speedup.n_trees + w.energy.n_trees
     return {"run_blocks_per_kernel": r["run_blocks"] / n, "runs_per_kernel_tree": r["runs"] / (n * max(trees, 1)),
@@ -225,11 +239,11 @@ def run_reference(args, rank, world):
     cfg = args.config
     n_k, n_f = W.CONFIGS[cfg][0], W.CONFIGS[cfg][1]
     cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
-    sp, en, freqs, d = W.make_models(cfg)
+    sp, en, freqs, d = bench_models(cfg, args.models)
     dec = decisions_per_eval(sp) + decisions_per_eval(en)
     # bounded sample: ~2 s of wall per step at ~6e7 decisions/s/core (calibrated below)
     ctx = mp.get_context("fork")
-    with ctx.Pool(cores, initializer=_pool_init, initargs=(cfg,)) as pool:
+    with ctx.Pool(cores, initializer=_pool_init, initargs=(cfg, args.models)) as pool:
         t = pool.map(_oracle_range, [(cfg, 0, 1, cfg)] * cores)
         per_kernel = max(min(t), 1e-4)
         sample = int(max(cores, min(n_k, 2.0 / per_kernel * cores)))
@@ -248,7 +262,7 @@ def run_reference(args, rank, world):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": workload_desc(cfg), "sample_kernels_per_step": sample,
+            "config": {"workload": workload_desc(cfg, args.models), "sample_kernels_per_step": sample,
                        "decisions_per_eval": dec},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": len(jobs), "kind": "oracle", "sample": desc},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -284,7 +298,7 @@ def main():
 
     cfg = args.config
     n_cfg, n_f = W.CONFIGS[cfg][0], W.CONFIGS[cfg][1]
-    sp_spec, en_spec, freqs, d = W.make_models(cfg)
+    sp_spec, en_spec, freqs, d = bench_models(cfg, args.models)
     targets = W.targets_six() if W.CONFIGS[cfg][4] == "six" else W.targets_es_pl()
     weak = args.scaling == "weak"
     if weak:
@@ -320,6 +334,8 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    syn.timing_read()                                       # drop anything recorded so far
+    syn.timing_enable(True)                                 # per-kernel events on the launch stream
     with sampler:
         for i in range(K):
             flush.zero_()                                   # L2 flush, outside the events
@@ -335,6 +351,8 @@ def main():
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
+    syn.timing_enable(False)
+    ktimes = syn.timing_read()                              # {kernel: (total ms, launches)}
     kern_ms = [a.elapsed_time(b) for a, b, _ in ev]
     step_ms = [a.elapsed_time(c) for a, _, c in ev]
     total_ms = sum(step_ms)
@@ -394,9 +412,12 @@ def main():
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     dec = decisions_per_eval(sp_spec) + decisions_per_eval(en_spec)
-    kern_avg_s = statistics.mean(kern_ms) / 1e3
-    variant = syn.last_launch()["variant"]
-    algo = {0: "k_sweep", 1: "k_sweep_iv", 2: "k_sweep_ws", 3: "k_sweep_da"}[variant // 1000 if variant >= 1000 else 0]
+    # dominant kernel of the step, timed by the library's events on its launch stream
+    algo = max(ktimes, key=lambda k: ktimes[k][0]) if ktimes else "k_sweep_da"
+    kern_avg_s = (ktimes[algo][0] / ktimes[algo][1] / 1e3) if ktimes else statistics.mean(kern_ms) / 1e3
+    kernel_share = ktimes[algo][0] / total_ms if ktimes else sum(kern_ms) / total_ms
+    per_kernel = {k: {"ms_per_launch": v[0] / v[1], "launches": v[1], "share_of_step": v[0] / total_ms}
+                  for k, v in ktimes.items()}
     hbm_bytes = evals_step // n_f * (W.N_STATIC * 4 + n_t * 4) + n_f * 4 + \
         sp.info()["device_bytes"] + en.info()["device_bytes"]
     hbm_ach = hbm_bytes / kern_avg_s / 1e9
@@ -404,16 +425,28 @@ def main():
            "algorithmic_bytes": hbm_bytes, "peak_source": peak_src}
     work = None
     if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws"):
-        work = run_walk_work(cfg, row0, n_local)
-    if work is not None:
+        work = run_walk_work(cfg, row0, n_local, which=args.models)
+    if algo == "k_svr":
+        # fp64 FMA-pipe roofline: 2 * n_k * n_f * n_SV flops per contraction
+        per_step = max(1.0, ktimes[algo][1] / K)              # kernel-slab launches per step
+        flops = 2.0 * (evals_step // n_f) * n_f * en_spec.n_sv / per_step
+        achieved = flops / kern_avg_s / 1e12
+        peak = 64 * 2 * sms * sm_max * 1e6 / 1e12
+        roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                    "traffic": None, "kernel": algo, "kernel_ms": kern_avg_s * 1e3,
+                    "kernel_share_of_step": kernel_share, "algorithmic_flops_per_launch": flops,
+                    "peak_note": f"fp64 FMA pipe 64 FMA/clk/SM x 2 x {sms} SMs x {sm_max:.0f} MHz (derived; "
+                                 "tcgen05 has no fp64 kind)",
+                    "hbm": hbm, "per_kernel": per_kernel}
+    elif work is not None:
         # on-chip L1 roofline: each run walk fetches max(1, ceil(depth/2)) 32-byte
         # 2-level blocks; counted by the oracle from the inputs (runs of clocks sharing a leaf)
         blocks = work["run_blocks_per_kernel"] * (evals_step // n_f)
         achieved = 32.0 * blocks / kern_avg_s / 1e9
         peak = 128.0 * sms * sm_max * 1e6 / 1e9
         roofline = {"bound": "l1", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                    "traffic": ncu_traffic(cfg), "kernel": algo, "kernel_ms": statistics.mean(kern_ms),
-                    "kernel_share_of_step": sum(kern_ms) / total_ms,
+                    "traffic": ncu_traffic(cfg) if args.models == "rf" else None, "kernel": algo,
+                    "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "algorithmic_bytes_per_launch": 32.0 * blocks,
                     "work": {"unit": "32-byte 2-level block fetches of the run walks", "per_launch": blocks,
                              "runs_per_kernel_tree": work["runs_per_kernel_tree"], "counted_on": work["sample"]},
@@ -424,19 +457,19 @@ def main():
                                         "note": "one 256-bit LDG (one 32-B sector, one L1 request) per block fetch; "
                                                 "peak = 1 scattered request per clk per SM"},
                     "decisions_per_s_vs_direct": evals_step * dec / kern_avg_s,
-                    "hbm": hbm}
+                    "hbm": hbm, "per_kernel": per_kernel}
     else:
         achieved = evals_step * dec / kern_avg_s / 1e9                  # G node-decisions / s
         peak = sms * sm_max * 1e6 * 32 / 2 / 1e9
         roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
-                    "frac": achieved / peak, "traffic": ncu_traffic(cfg), "kernel": algo,
-                    "kernel_ms": statistics.mean(kern_ms), "kernel_share_of_step": sum(kern_ms) / total_ms,
+                    "frac": achieved / peak, "traffic": ncu_traffic(cfg) if args.models == "rf" else None,
+                    "kernel": algo, "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
-                    "hbm": hbm}
+                    "hbm": hbm, "per_kernel": per_kernel}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, ev_n, el = oracle_single_core(cfg, min(n_cfg, 1000))
+        v, ev_n, el = oracle_single_core(cfg, min(n_cfg, 1000), which=args.models)
         cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"first {min(n_cfg, 1000)} kernels of {cfg} x {n_f} clocks repeated to "
                          f"{el:.1f} s ({ev_n} evals), single-threaded oracle (oracle/oracle.c)"}
@@ -446,7 +479,7 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
                 "warmup": args.warmup, "ms_per_step": total_ms_max / K, "higher_is_better": True,
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": workload_desc(cfg), "n_kernels_per_rank": n_local,
+                "config": {"workload": workload_desc(cfg, args.models), "n_kernels_per_rank": n_local,
                            "n_freqs": n_f, "targets": n_t,
                            "parallelism": f"dp{world} (kernel axis) + NCCL all-gather of choices",
                            "l2": f"flushed between timed steps ({args.flush_mib} MiB write)",

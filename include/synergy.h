@@ -90,10 +90,11 @@ typedef void *syn_stream;   /* cudaStream_t */
  * clock part, so the device evaluates sum_j (dual_j e^{-gamma A_kj}) e^{-gamma B_ji}: a
  * [kernels x SVs] x [SVs x clocks] fp64 contraction (Q24).  It agrees with the plain
  * definition within 2^-40 * (|svr_intercept| + sum_j |dual_coef[j]|), NOT bit for bit.
- * Calls whose models have an SVR member take scratch of (n_sv + splits * n_kernels) * n_freqs
- * * 8 bytes per SVR model from the device's default stream-ordered memory pool
- * (cudaMallocAsync / cudaFreeAsync on the call's stream; splits <= 16), the only allocation a
- * hot call makes. */
+ * Calls whose models have an SVR member take stream-ordered scratch per SVR model of about
+ * (n_sv * (n_freqs + min(n_kernels, 2^25 / n_sv)) + splits * n_kernels * n_freqs) * 8 bytes
+ * (splits <= 16) from a library-owned CUDA memory pool on the device (cudaMallocFromPoolAsync /
+ * cudaFreeAsync on the call's stream; the pool keeps freed memory mapped, so after the first
+ * call of a given size no device memory is mapped), the only allocation a hot call makes. */
 typedef struct {
     int32_t n_inputs;            /* F + 1, 1 .. SYNERGY_MAX_INPUTS                        */
     double linear_weight;        /* 0 => no linear member                                 */
@@ -234,6 +235,16 @@ syn_status synergy_sweep_host(syn_workspace *ws, const syn_model *speedup,
  * benchmarks: kernels launched, evaluations, node decisions of complete paths).  NULLs ok. */
 syn_status synergy_last_launch(int32_t *kernels_launched, int64_t *evals, int64_t *grid,
                                int32_t *block, int32_t *variant);
+
+/* Per-kernel device timing for measurement (bench.py's roofline).  While enabled, every library
+ * kernel launch is bracketed by two CUDA events recorded on its launch stream (two extra stream
+ * operations per launch; off by default).  synergy_timing_read synchronises the recorded events,
+ * sums the elapsed time per kernel name since the previous read, clears the record and returns
+ * up to `cap` entries: names[k] (static strings, e.g. "k_sweep_da", "k_svr"), total_ms[k],
+ * launches[k]; *n_kernels = number of distinct kernels recorded.  Process-wide, thread-safe. */
+syn_status synergy_timing_enable(int32_t on);
+syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms, int64_t *launches,
+                               int32_t *n_kernels);
 
 #ifdef __cplusplus
 }

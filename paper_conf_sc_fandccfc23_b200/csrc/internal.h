@@ -56,10 +56,12 @@ struct DevModel {
     int svr_splits;
 };
 
-// k_svr tiling: 8 warps x kSvrRows kernels per CTA, 32 x CPT clocks, SVs staged kSvrJC at a time
+// SVR contraction tiling (kernels_svr.cuh): 8 warps x kSvrRows kernels = kSvrTK kernels per CTA,
+// 32 x CPT clocks, SVs staged kSvrJC at a time through a kSvrStages-deep bulk-copy ring
 constexpr int kSvrRows = 8;
 constexpr int kSvrTK = 8 * kSvrRows;
 constexpr int kSvrJC = 16;
+constexpr int kSvrStages = 3;
 constexpr int kSvrMaxSplits = 16;
 
 struct SvrArgs {
@@ -68,15 +70,20 @@ struct SvrArgs {
     int F;
     const float* freqs;      // [n_f]
     int n_f;
-    const float* sv;
+    const float* sv;         // [n_sv][F + 1]
     const double* dual;
     const double* in_mean;
     const double* in_scale;
     double gamma;
     int n_sv;
-    int sv_per_split;        // SV range of split blockIdx.z
-    double* V;               // [n_sv][n_f] clock factors e^{-gamma B_ji}
-    double* P;               // [splits][n_k][n_f]
+    int n_svp;               // n_sv rounded up to kSvrJC (padding rows are zero)
+    int tn;                  // clock tile (32 * CPT)
+    int chunks_per_split;    // kSvrJC-SV chunks per split (blockIdx.z)
+    long long slab0;         // first kernel of this slab
+    int nks;                 // kernels in this slab
+    double* Ut;              // [ceil(nks / kSvrTK)][n_svp][kSvrTK]   U_kj = dual_j e^{-gamma A_kj}
+    double* Vt;              // [ceil(n_f / tn)][n_svp][tn]           V_ji = e^{-gamma B_ji}
+    double* P;               // [splits][n_k][n_f] partial contractions
 };
 
 constexpr int kMaxTargets = 16;

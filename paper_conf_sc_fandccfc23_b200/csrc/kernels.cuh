@@ -106,18 +106,13 @@ __device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
     }
 }
 
-// One warp selects all targets of one kernel from its n_f normalised predictions
-// (S, E in shared or global memory).  Writes out[0..n_t).
-__device__ __forceinline__ void select_row_warp(const float* S, const float* E, const float* P2,
-                                                const float* P3, int n_f, int def,
-                                                int n_t, const int* kind, const float* xs,
-                                                int* out, int lane) {
+// Selection baselines of one row (Q14-Q16): returns false if the default clock's
+// prediction is invalid (every target then -1); else E_def, S_def and the minimum-energy point's
+// E_min, S_minE (lowest index among equal minima, L265).  Whole warp, result in every lane.
+__device__ __forceinline__ bool select_baseline(const float* S, const float* E, int n_f, int def, int lane,
+                                                double& E_def, double& S_def, double& E_min, double& S_minE) {
     const float sd = S[def], ed = E[def];
-    if (!valid_pred(sd, ed)) {              // no baseline: every target -1
-        for (int t = lane; t < n_t; t += 32) out[t] = -1;
-        return;
-    }
-    // minimum-energy point, lowest index among equal minima (baseline of ES/PL, L265)
+    if (!valid_pred(sd, ed)) return false;
     double be = CUDART_INF;
     int bi = INT_MAX;
     for (int i = lane; i < n_f; i += 32) {
@@ -125,103 +120,126 @@ __device__ __forceinline__ void select_row_warp(const float* S, const float* E, 
         if (valid_pred(s, e) && (double)e < be) { be = (double)e; bi = i; }
     }
     argmin_shfl(be, bi);
-    const double E_def = (double)ed, S_def = (double)sd;
-    const double E_min = (double)E[bi], S_minE = (double)S[bi];
+    E_def = (double)ed;
+    S_def = (double)sd;
+    E_min = (double)E[bi];
+    S_minE = (double)S[bi];
+    return true;
+}
+
+// One target of one row: the lowest index minimising the target's key
+// among valid feasible clocks, -1 if none.  P2/P3: direct EDP / ED2P predictions or null.
+__device__ __forceinline__ int select_target(const float* S, const float* E, const float* P2, const float* P3,
+                                             int n_f, int kd, float x, double E_def, double S_def,
+                                             double E_min, double S_minE, int lane) {
+    const double frac = __ddiv_rn((double)x, 100.0);
+    const double thr_es = __dsub_rn(E_def, __dmul_rn(frac, __dsub_rn(E_def, E_min)));
+    const double thr_pl = __dsub_rn(S_def, __dmul_rn(frac, __dsub_rn(S_def, S_minE)));
+    double bk = CUDART_INF;
+    int bx = INT_MAX;
+    for (int i = lane; i < n_f; i += 32) {
+        const float sf = S[i], ef = E[i];
+        if (!valid_pred(sf, ef)) continue;
+        const double s = (double)sf, e = (double)ef;
+        double key;
+        bool feas = true;
+        switch (kd) {
+            case 0: key = -s; break;                                   // MAX_PERF
+            case 1: key = e; break;                                    // MIN_ENERGY
+            case 2:                                                    // MIN_EDP  e*t
+                if (P2) { const float p = P2[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
+                else key = __ddiv_rn(e, s);
+                break;
+            case 3:                                                    // MIN_ED2P e*t^2
+                if (P3) { const float p = P3[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
+                else key = __ddiv_rn(__ddiv_rn(e, s), s);
+                break;
+            case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
+            default: feas = (s >= thr_pl); key = e; break;             // PL_x
+        }
+        if (feas && (key < bk || (key == bk && i < bx))) { bk = key; bx = i; }
+    }
+    argmin_shfl(bk, bx);
+    return bx == INT_MAX ? -1 : bx;
+}
+
+// Every target of one row, one warp (standalone selection and the choice-error truth).
+__device__ __forceinline__ void select_row_warp(const float* S, const float* E, const float* P2,
+                                                const float* P3, int n_f, int def,
+                                                int n_t, const int* kind, const float* xs,
+                                                int* out, int lane) {
+    double E_def, S_def, E_min, S_minE;
+    if (!select_baseline(S, E, n_f, def, lane, E_def, S_def, E_min, S_minE)) {
+        for (int t = lane; t < n_t; t += 32) out[t] = -1;
+        return;
+    }
     for (int t = 0; t < n_t; ++t) {
-        const int kd = kind[t];
-        const double frac = __ddiv_rn((double)xs[t], 100.0);
-        const double thr_es = __dsub_rn(E_def, __dmul_rn(frac, __dsub_rn(E_def, E_min)));
-        const double thr_pl = __dsub_rn(S_def, __dmul_rn(frac, __dsub_rn(S_def, S_minE)));
-        double bk = CUDART_INF;
-        int bx = INT_MAX;
-        for (int i = lane; i < n_f; i += 32) {
-            const float sf = S[i], ef = E[i];
-            if (!valid_pred(sf, ef)) continue;
-            const double s = (double)sf, e = (double)ef;
-            double key;
-            bool feas = true;
-            switch (kd) {
-                case 0: key = -s; break;                                   // MAX_PERF
-                case 1: key = e; break;                                    // MIN_ENERGY
-                case 2:                                                    // MIN_EDP  e*t
-                    if (P2) { const float p = P2[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
-                    else key = __ddiv_rn(e, s);
-                    break;
-                case 3:                                                    // MIN_ED2P e*t^2
-                    if (P3) { const float p = P3[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
-                    else key = __ddiv_rn(__ddiv_rn(e, s), s);
-                    break;
-                case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
-                default: feas = (s >= thr_pl); key = e; break;             // PL_x
-            }
-            if (feas && (key < bk || (key == bk && i < bx))) { bk = key; bx = i; }
-        }
-        argmin_shfl(bk, bx);
-        if (lane == 0) out[t] = (bx == INT_MAX) ? -1 : bx;
+        const int c = select_target(S, E, P2, P3, n_f, kind[t], xs[t], E_def, S_def, E_min, S_minE, lane);
+        if (lane == 0) out[t] = c;
     }
 }
 
-// Per kernel of the tile (one warp each): normalise the raw fp64 model outputs to the default
-// clock (S = (float)(mS_i / mS_def), L69 / DESIGN.md Q13; raw (float)m when def == -1), write
-// the predictions if requested, then run the per-target selection.  mS/mE: [nk][n_f] doubles,
-// sS/sE: [nk][n_f] float scratch, all in shared memory.  Caller has synchronised the block.
-__device__ __forceinline__ void finish_tile(const SweepArgs& a, double* mS, double* mE,
-                                            float* sS, float* sE, int nk, long long k0) {
-    const int n_f = a.n_f;
-    const int lane = threadIdx.x & 31;
-    const int nw = blockDim.x >> 5;
-    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
-        double* rS = mS + (size_t)kl * n_f;
-        double* rE = mE + (size_t)kl * n_f;
-        float* oS = sS + (size_t)kl * n_f;
-        float* oE = sE + (size_t)kl * n_f;
-        const long long k = k0 + kl;
-        add_svr_row(a.ms, rS, k, a.n_k, n_f, lane);       // SVR member last (ensemble order, Q7)
-        add_svr_row(a.me, rE, k, a.n_k, n_f, lane);
-        const double dS = a.def >= 0 ? rS[a.def] : 1.0;
-        const double dE = a.def >= 0 ? rE[a.def] : 1.0;
-        for (int i = lane; i < n_f; i += 32) {
-            const float s = a.def >= 0 ? __double2float_rn(__ddiv_rn(rS[i], dS)) : __double2float_rn(rS[i]);
-            const float e = a.def >= 0 ? __double2float_rn(__ddiv_rn(rE[i], dE)) : __double2float_rn(rE[i]);
-            oS[i] = s;
-            oE[i] = e;
-            if (a.S_out) a.S_out[k * n_f + i] = s;
-            if (a.E_out) a.E_out[k * n_f + i] = e;
-        }
-        __syncwarp();
-        if (a.mode == kModeSweep)
-            select_row_warp(oS, oE, nullptr, nullptr, n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
-    }
-}
-
-// finish_tile for the four-model variant: mv[m] / sv[m] ([nk][n_f]) for models m < 4 (mv[m] null
-// when absent); direct EDP / ED2P predictions become the MIN_EDP / MIN_ED2P keys.
+// Finish of a tile of nk kernels (all threads of the CTA; caller has synchronised the block).
+// mv[m] ([nk][n_f] fp64 raw outputs in shared memory) for models m < 4 — speedup, energy,
+// direct EDP, direct ED2P; mv[m] null when absent — and sv[m] the matching float scratch.
+//   1. SVR members (add_svr_row's arithmetic), every (row, clock) in parallel
+//   2. normalise to the default clock (S = (float)(m_i / m_def), L69 / DESIGN.md Q13; raw
+//      (float)m when def == -1), write the predictions if requested
+//   3. per (row, target) one warp: baselines + the target's argmin; direct EDP / ED2P
+//      predictions become the MIN_EDP / MIN_ED2P keys
 __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* mv, float* const* sv,
                                              int nk, long long k0) {
     const int n_f = a.n_f;
     const int lane = threadIdx.x & 31;
     const int nw = blockDim.x >> 5;
-    for (int kl = threadIdx.x >> 5; kl < nk; kl += nw) {
-        const long long k = k0 + kl;
-        for (int m = 0; m < 4; ++m) {
-            if (!mv[m]) continue;
-            double* r = mv[m] + (size_t)kl * n_f;
-            add_svr_row(m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2], r, k, a.n_k, n_f, lane);
-            float* o = sv[m] + (size_t)kl * n_f;
-            float* g = m == 0 ? a.S_out : m == 1 ? a.E_out : a.X_out[m - 2];
-            const double dv = a.def >= 0 ? r[a.def] : 1.0;
-            for (int i = lane; i < n_f; i += 32) {
-                const float v = a.def >= 0 ? __double2float_rn(__ddiv_rn(r[i], dv)) : __double2float_rn(r[i]);
-                o[i] = v;
-                if (g) g[k * n_f + i] = v;
-            }
+    const int units = nk * n_f;
+    bool any_svr = false;
+    for (int m = 0; m < 4; ++m) {
+        if (!mv[m]) continue;
+        const DevModel& md = m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+        if (md.svr_weight == 0.0) continue;
+        any_svr = true;
+        for (int u = threadIdx.x; u < units; u += blockDim.x) {
+            const int kl = u / n_f;
+            add_svr_unit(md, mv[m] + u, k0 + kl, a.n_k, n_f, u - kl * n_f);
         }
-        __syncwarp();
-        if (a.mode == kModeSweep)
-            select_row_warp(sv[0] + (size_t)kl * n_f, sv[1] + (size_t)kl * n_f,
-                            mv[2] ? sv[2] + (size_t)kl * n_f : nullptr, mv[3] ? sv[3] + (size_t)kl * n_f : nullptr,
-                            n_f, a.def, a.n_t, a.kind, a.x, a.choice + k * a.n_t, lane);
     }
+    if (any_svr) __syncthreads();
+    for (int m = 0; m < 4; ++m) {
+        if (!mv[m]) continue;
+        float* g = m == 0 ? a.S_out : m == 1 ? a.E_out : a.X_out[m - 2];
+        for (int u = threadIdx.x; u < units; u += blockDim.x) {
+            const int kl = u / n_f;
+            const double* r = mv[m] + (size_t)kl * n_f;
+            const double v64 = mv[m][u];
+            const float v = a.def >= 0 ? __double2float_rn(__ddiv_rn(v64, r[a.def])) : __double2float_rn(v64);
+            sv[m][u] = v;
+            if (g) g[k0 * n_f + u] = v;
+        }
+    }
+    if (a.mode != kModeSweep) return;
+    __syncthreads();
+    const int n_t = a.n_t;
+    for (int task = threadIdx.x >> 5; task < nk * n_t; task += nw) {
+        const int kl = task / n_t, t = task - kl * n_t;
+        const float* S = sv[0] + (size_t)kl * n_f;
+        const float* E = sv[1] + (size_t)kl * n_f;
+        double E_def, S_def, E_min, S_minE;
+        int c = -1;
+        if (select_baseline(S, E, n_f, a.def, lane, E_def, S_def, E_min, S_minE))
+            c = select_target(S, E, mv[2] ? sv[2] + (size_t)kl * n_f : nullptr,
+                              mv[3] ? sv[3] + (size_t)kl * n_f : nullptr, n_f, a.kind[t], a.x[t],
+                              E_def, S_def, E_min, S_minE, lane);
+        if (lane == 0) a.choice[(k0 + kl) * n_t + t] = c;
+    }
+}
+
+// Two-model finish (speedup, energy).
+__device__ __forceinline__ void finish_tile(const SweepArgs& a, double* mS, double* mE,
+                                            float* sS, float* sE, int nk, long long k0) {
+    double* mv[4] = {mS, mE, nullptr, nullptr};
+    float* sv[4] = {sS, sE, nullptr, nullptr};
+    finish_tile4(a, mv, sv, nk, k0);
 }
 
 template <int SLOTS, int TILP>

@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <string>
 #include <vector>
@@ -60,6 +61,54 @@ struct LaunchInfo {
     int variant;
 };
 thread_local LaunchInfo g_last = {0, 0, 0, 0, 0};
+
+// Optional per-kernel device timing (synergy_timing_enable): CUDA events recorded on the launch
+// stream around every library kernel launch; read back (summed per kernel) by synergy_timing_read.
+struct TimedLaunch {
+    const char* name;
+    cudaEvent_t a, b;
+};
+std::mutex g_tmu;
+bool g_timing = false;
+std::vector<TimedLaunch> g_tl;
+std::vector<cudaEvent_t> g_evpool;
+
+cudaEvent_t take_event() {
+    if (!g_evpool.empty()) {
+        cudaEvent_t e = g_evpool.back();
+        g_evpool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    if (cudaEventCreate(&e) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return e;
+}
+
+struct KernelTimer {   // records around one launch when timing is enabled
+    const char* name;
+    cudaStream_t st;
+    cudaEvent_t a = nullptr;
+    KernelTimer(const char* n, cudaStream_t s) : name(n), st(s) {
+        std::lock_guard<std::mutex> lock(g_tmu);
+        if (!g_timing) return;
+        a = take_event();
+        if (a) cudaEventRecord(a, st);
+    }
+    ~KernelTimer() {
+        if (!a) return;
+        std::lock_guard<std::mutex> lock(g_tmu);
+        cudaEvent_t b = take_event();
+        if (!b) {
+            g_evpool.push_back(a);
+            return;
+        }
+        cudaEventRecord(b, st);
+        g_tl.push_back({name, a, b});
+    }
+};
 
 syn_status fail(syn_status st, const char* fmt, ...) {
     char buf[512];
@@ -366,6 +415,33 @@ syn_status validate_sweep(const syn_model* sp, const syn_model* en, int64_t n_k,
     return SYN_OK;
 }
 
+// Library-owned stream-ordered pool per device for the SVR scratch: memory freed with
+// cudaFreeAsync stays mapped (release threshold = max), so steady-state calls reuse it instead
+// of remapping; the process's default pool and its settings are left alone.
+cudaMemPool_t svr_pool(int dev) {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    if (dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lock(mu);
+    if (!pools[dev]) {
+        cudaMemPoolProps props;
+        memset(&props, 0, sizeof props);
+        props.allocType = cudaMemAllocationTypePinned;
+        props.handleTypes = cudaMemHandleTypeNone;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        unsigned long long thr = ~0ULL;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = p;
+    }
+    return pools[dev];
+}
+
 // SVR members (kernels_svr.cuh): per model, V = clock factors and the split contractions P into
 // stream-ordered scratch; dm.svr_p / svr_splits point the finish step at them.  Released with
 // release() after the sweep kernel is enqueued (cudaFreeAsync keeps it alive until then).
@@ -381,16 +457,19 @@ struct SvrScratch {
 };
 
 template <int CPT>
-cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, size_t smem, cudaStream_t st) {
-    static size_t smem_set = 48 * 1024;
-    if (smem > smem_set) {
+cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, cudaStream_t st) {
+    static bool smem_set = false;
+    const size_t smem = (size_t)kSvrStages * kSvrJC * (kSvrTK + 32 * CPT) * sizeof(double) + kSvrStages * 8;
+    if (!smem_set) {
         cudaError_t e = cudaFuncSetAttribute(k_svr<CPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        smem_set = smem;
+        smem_set = true;
     }
     k_svr<CPT><<<grid, 256, smem, st>>>(sa);
     return cudaGetLastError();
 }
+
+constexpr size_t kSvrSlabBytes = 256u << 20;   // U scratch per kernel slab
 
 syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
                        cudaStream_t st, SvrScratch& scr) {
@@ -399,25 +478,34 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     const int n_f = clocks->n_f;
     const int cpt = std::min(8, (n_f + 31) / 32);
     const int tn = 32 * cpt;
-    const long long tiles_n = (n_f + tn - 1) / tn;
-    const long long tiles = (n_k + kSvrTK - 1) / kSvrTK * tiles_n;
-    if ((n_k + kSvrTK - 1) / kSvrTK > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for k_svr");
+    const int tiles_n = (n_f + tn - 1) / tn;
+    const int n_svp = (dm.n_sv + kSvrJC - 1) / kSvrJC * kSvrJC;
+    const int n_chunks = n_svp / kSvrJC;
+    // kernel slabs bound the U scratch; each slab is one k_svr_u + one k_svr launch
+    long long nks = std::max<long long>(kSvrTK, (long long)(kSvrSlabBytes / ((size_t)n_svp * 8)) / kSvrTK * kSvrTK);
+    nks = std::min<long long>(nks, (n_k + kSvrTK - 1) / kSvrTK * kSvrTK);
+    const long long tiles = (std::min(nks, n_k) + kSvrTK - 1) / kSvrTK * tiles_n;
+    if ((nks + kSvrTK - 1) / kSvrTK > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for k_svr");
     // split the SV range across CTAs until the grid covers the SMs (at most kSvrMaxSplits)
-    long long splits = std::max<long long>(1, sm_count(device) / std::max<long long>(tiles, 1));
-    splits = std::min<long long>(splits, kSvrMaxSplits);
-    splits = env_int("SYNERGY_SVR_SPLITS", (int)splits);
-    splits = std::max<long long>(1, std::min<long long>(splits, (dm.n_sv + kSvrJC - 1) / kSvrJC));
-    const int per = (int)(((dm.n_sv + splits - 1) / splits + kSvrJC - 1) / kSvrJC * kSvrJC);
-    splits = (dm.n_sv + per - 1) / per;
-    const size_t vb = (size_t)dm.n_sv * n_f * sizeof(double);
+    int splits = (int)std::max<long long>(1, sm_count(device) / std::max<long long>(tiles, 1));
+    splits = std::min(splits, kSvrMaxSplits);
+    splits = env_int("SYNERGY_SVR_SPLITS", splits);
+    splits = std::max(1, std::min(splits, n_chunks));
+    const int cps = (n_chunks + splits - 1) / splits;
+    splits = (n_chunks + cps - 1) / cps;
     const size_t pb = (size_t)splits * (size_t)n_k * n_f * sizeof(double);
-    const size_t voff = (pb + 255) / 256 * 256;
+    const size_t vb = (size_t)tiles_n * n_svp * tn * sizeof(double);
+    const size_t ub = (size_t)((nks + kSvrTK - 1) / kSvrTK) * n_svp * kSvrTK * sizeof(double);
+    const size_t voff = (pb + 255) / 256 * 256, uoff = voff + (vb + 255) / 256 * 256;
+    const size_t total = uoff + ub;
     void* buf = nullptr;
-    cudaError_t e = cudaMallocAsync(&buf, voff + vb, st);
+    cudaMemPool_t pool = svr_pool(device);
+    if (!pool) return fail(SYN_ERR_CUDA, "cannot create the SVR scratch pool on device %d", device);
+    cudaError_t e = cudaMallocFromPoolAsync(&buf, total, pool, st);
     if (e != cudaSuccess) {
         cudaGetLastError();
-        return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "SVR scratch of %zu bytes", voff + vb)
-                                              : cuda_fail(e, "cudaMallocAsync(SVR scratch)");
+        return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "SVR scratch of %zu bytes", total)
+                                              : cuda_fail(e, "cudaMallocFromPoolAsync(SVR scratch)");
     }
     scr.bufs.push_back(buf);
     SvrArgs sa;
@@ -433,28 +521,54 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     sa.in_scale = dm.in_scale;
     sa.gamma = dm.svr_gamma;
     sa.n_sv = dm.n_sv;
-    sa.sv_per_split = per;
+    sa.n_svp = n_svp;
+    sa.tn = tn;
+    sa.chunks_per_split = cps;
     sa.P = static_cast<double*>(buf);
-    sa.V = reinterpret_cast<double*>(static_cast<char*>(buf) + voff);
-    const long long nv = (long long)dm.n_sv * n_f;
-    k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
-    if ((e = cudaGetLastError()) != cudaSuccess) return cuda_fail(e, "k_svr_v launch");
-    const size_t smem = ((size_t)F * kSvrTK + (size_t)kSvrJC * kSvrTK + (size_t)kSvrJC * tn) * sizeof(double);
-    const dim3 grid((unsigned)((n_k + kSvrTK - 1) / kSvrTK), (unsigned)tiles_n, (unsigned)splits);
-    switch (cpt) {
-        case 1: e = launch_svr_t<1>(sa, grid, smem, st); break;
-        case 2: e = launch_svr_t<2>(sa, grid, smem, st); break;
-        case 3: e = launch_svr_t<3>(sa, grid, smem, st); break;
-        case 4: e = launch_svr_t<4>(sa, grid, smem, st); break;
-        case 5: e = launch_svr_t<5>(sa, grid, smem, st); break;
-        case 6: e = launch_svr_t<6>(sa, grid, smem, st); break;
-        case 7: e = launch_svr_t<7>(sa, grid, smem, st); break;
-        default: e = launch_svr_t<8>(sa, grid, smem, st); break;
+    sa.Vt = reinterpret_cast<double*>(static_cast<char*>(buf) + voff);
+    sa.Ut = reinterpret_cast<double*>(static_cast<char*>(buf) + uoff);
+    const long long nv = (long long)tiles_n * n_svp * tn;
+    {
+        KernelTimer kt("k_svr_v", st);
+        k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
+        e = cudaGetLastError();
     }
-    if (e != cudaSuccess) return cuda_fail(e, "k_svr launch");
-    scr.launches += 2;
+    if (e != cudaSuccess) return cuda_fail(e, "k_svr_v launch");
+    scr.launches += 1;
+    static bool u_smem_set = false;
+    const size_t usmem = (size_t)F * (64 * sizeof(double) + kSvrJC * sizeof(float));
+    if (usmem > 48 * 1024 && !u_smem_set) {
+        if ((e = cudaFuncSetAttribute(k_svr_u, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024)) != cudaSuccess)
+            return cuda_fail(e, "k_svr_u attribute");
+        u_smem_set = true;
+    }
+    for (long long s0 = 0; s0 < n_k; s0 += nks) {
+        sa.slab0 = s0;
+        sa.nks = (int)std::min<long long>(nks, n_k - s0);
+        const unsigned kts = (unsigned)((sa.nks + kSvrTK - 1) / kSvrTK);
+        {
+            KernelTimer kt("k_svr_u", st);
+            k_svr_u<<<dim3(kts, (unsigned)(n_svp / kSvrJC)), 256, usmem, st>>>(sa);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "k_svr_u launch");
+        const dim3 grid(kts, (unsigned)tiles_n, (unsigned)splits);
+        KernelTimer kt("k_svr", st);
+        switch (cpt) {
+            case 1: e = launch_svr_t<1>(sa, grid, st); break;
+            case 2: e = launch_svr_t<2>(sa, grid, st); break;
+            case 3: e = launch_svr_t<3>(sa, grid, st); break;
+            case 4: e = launch_svr_t<4>(sa, grid, st); break;
+            case 5: e = launch_svr_t<5>(sa, grid, st); break;
+            case 6: e = launch_svr_t<6>(sa, grid, st); break;
+            case 7: e = launch_svr_t<7>(sa, grid, st); break;
+            default: e = launch_svr_t<8>(sa, grid, st); break;
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "k_svr launch");
+        scr.launches += 2;
+    }
     dm.svr_p = sa.P;
-    dm.svr_splits = (int)splits;
+    dm.svr_splits = splits;
     return ok();
 }
 
@@ -529,10 +643,15 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     syn_status ss = prepare_svr(a.ms, clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss == SYN_OK) ss = prepare_svr(a.me, clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss != SYN_OK) return ss;
-    cudaError_t e = c.algo == 3 ? launch_da(a, c, grid, st)
+    static const char* knames[4] = {"k_sweep", "k_sweep_iv", "k_sweep_ws", "k_sweep_da"};
+    cudaError_t e;
+    {
+        KernelTimer kt(knames[c.algo], st);
+        e = c.algo == 3 ? launch_da(a, c, grid, st)
                   : c.algo == 2 ? launch_ws(a, c, grid, st)
                   : c.algo == 1 ? launch_iv(a, c, grid, st)
                                 : launch_sweep(a, c, grid, st);
+    }
     static const char* names[4] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch", "k_sweep_da launch"};
     if (e != cudaSuccess) return cuda_fail(e, names[c.algo]);
     g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
@@ -957,7 +1076,11 @@ syn_status synergy_sweep4(const syn_model* const* models, const float* d_feature
     for (int m = 0; m < 4 && ss == SYN_OK; ++m)
         if (m < 2 || a.has_x[m - 2]) ss = prepare_svr(*dms[m], clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss != SYN_OK) return ss;
-    cudaError_t e = launch_da(a, c, grid, st);
+    cudaError_t e;
+    {
+        KernelTimer kt("k_sweep_da", st);
+        e = launch_da(a, c, grid, st);
+    }
     if (e != cudaSuccess) return cuda_fail(e, "k_sweep_da launch");
     g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, 3000 + c.tile_k};
     return ok();
@@ -993,7 +1116,10 @@ syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32
     const int block = 256;
     const long long need = (n_k + 7) / 8;
     const long long grid = std::min<long long>(need, (long long)sm_count(dev) * 8);
-    k_select<<<(unsigned)grid, block, 0, static_cast<cudaStream_t>(stream)>>>(a);
+    {
+        KernelTimer kt("k_select", static_cast<cudaStream_t>(stream));
+        k_select<<<(unsigned)grid, block, 0, static_cast<cudaStream_t>(stream)>>>(a);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "k_select launch");
     g_last = {1, n_k * (long long)n_f, grid, block, 0};
@@ -1128,6 +1254,44 @@ syn_status synergy_sweep_host(syn_workspace* w, const syn_model* sp, const syn_m
     if (n_k > 0 && (e = cudaMemcpyAsync(h_choice, w->d_choice, cb, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
         return cuda_fail(e, "cudaMemcpyAsync D2H");
     return ok();
+}
+
+syn_status synergy_timing_enable(int32_t on) {
+    std::lock_guard<std::mutex> lock(g_tmu);
+    g_timing = on != 0;
+    return ok();
+}
+
+syn_status synergy_timing_read(int32_t cap, const char** names, double* total_ms, int64_t* launches,
+                               int32_t* n_kernels) {
+    if (cap < 0 || (cap > 0 && (!names || !total_ms || !launches)) || !n_kernels)
+        return fail(SYN_ERR_INVALID_ARG, "bad timing_read buffers");
+    std::lock_guard<std::mutex> lock(g_tmu);
+    std::vector<const char*> nm;
+    std::vector<double> ms;
+    std::vector<int64_t> cnt;
+    syn_status st = SYN_OK;
+    for (const TimedLaunch& t : g_tl) {
+        float x = 0.0f;
+        cudaError_t e = cudaEventSynchronize(t.b);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&x, t.a, t.b);
+        if (e != cudaSuccess && st == SYN_OK) st = cuda_fail(e, "timing events");
+        size_t k = 0;
+        while (k < nm.size() && strcmp(nm[k], t.name)) ++k;
+        if (k == nm.size()) { nm.push_back(t.name); ms.push_back(0.0); cnt.push_back(0); }
+        ms[k] += x;
+        cnt[k] += 1;
+        g_evpool.push_back(t.a);
+        g_evpool.push_back(t.b);
+    }
+    g_tl.clear();
+    *n_kernels = (int32_t)nm.size();
+    for (int32_t k = 0; k < (int32_t)nm.size() && k < cap; ++k) {
+        names[k] = nm[k];
+        total_ms[k] = ms[k];
+        launches[k] = cnt[k];
+    }
+    return st == SYN_OK ? ok() : st;
 }
 
 syn_status synergy_last_launch(int32_t* kernels, int64_t* evals, int64_t* grid, int32_t* block, int32_t* variant) {

@@ -81,6 +81,8 @@ def load(path: str = LIB_PATH) -> C.CDLL:
         "synergy_workspace_destroy": (I32, [P]),
         "synergy_sweep_host": (I32, [P, P, P, P, I64, I32, P, I32, P, I32, P, P]),
         "synergy_last_launch": (I32, [P, P, P, P, P]),
+        "synergy_timing_enable": (I32, [I32]),
+        "synergy_timing_read": (I32, [I32, P, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -346,3 +348,18 @@ def last_launch():
     e, g = C.c_int64(), C.c_int64()
     _check(load().synergy_last_launch(C.byref(k), C.byref(e), C.byref(g), C.byref(b), C.byref(v)))
     return {"kernels": k.value, "evals": e.value, "grid": g.value, "block": b.value, "variant": v.value}
+
+
+def timing_enable(on: bool = True):
+    """synergy_timing_enable: bracket every library kernel launch with CUDA events."""
+    _check(load().synergy_timing_enable(1 if on else 0))
+
+
+def timing_read(cap: int = 32):
+    """synergy_timing_read: {kernel name: (total_ms, launches)} since the previous read."""
+    names = (C.c_char_p * cap)()
+    ms = (C.c_double * cap)()
+    cnt = (C.c_int64 * cap)()
+    n = C.c_int32()
+    _check(load().synergy_timing_read(cap, names, ms, cnt, C.byref(n)))
+    return {names[k].decode(): (ms[k], cnt[k]) for k in range(min(n.value, cap))}

@@ -1,5 +1,6 @@
 """Time the SVR path (k_svr_v + k_svr + finish) on config shapes: speedup linear, energy SVR."""
-import sys, json
+import os, sys, json
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
 import torch
 from paper_conf_sc_fandccfc23_b200 import synergy as syn, workloads as W
