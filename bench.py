@@ -224,7 +224,8 @@ def run_walk_work(cfg, row0, n_rows, budget=5e8, which="rf"):
     w = W.make_config(cfg, row0=row0, n=n, models=models)
     r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
     trees = w.speedup.n_trees + w.energy.n_trees
-    return {"run_blocks_per_kernel": r["run_blocks"] / n, "runs_per_kernel_tree": r["runs"] / (n * max(trees, 1)),
+    return {"run_blocks_per_kernel": r["run_blocks"] / n, "resume_blocks_per_kernel": r["resume_blocks"] / n,
+            "runs_per_kernel_tree": r["runs"] / (n * max(trees, 1)),
             "sample": f"rows [{row0}, {row0 + n}) of {cfg}" + (" (all launched rows)" if n == n_rows else
                                                              f" scaled to {n_rows} rows")}
 
@@ -424,7 +425,7 @@ def main():
     hbm = {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": hbm_ach / peaks["hbm_gbs"],
            "algorithmic_bytes": hbm_bytes, "peak_source": peak_src}
     work = None
-    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws"):
+    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws", "k_tm_walk"):
         work = run_walk_work(cfg, row0, n_local, which=args.models)
     if algo == "k_svr":
         # fp64 FMA-pipe roofline: 2 * n_k * n_f * n_SV flops per contraction
@@ -441,14 +442,19 @@ def main():
     elif work is not None:
         # on-chip L1 roofline: each run walk fetches max(1, ceil(depth/2)) 32-byte
         # 2-level blocks; counted by the oracle from the inputs (runs of clocks sharing a leaf)
-        blocks = work["run_blocks_per_kernel"] * (evals_step // n_f)
+        per_launch = max(1.0, ktimes[algo][1] / K)             # kernel-slab launches per step
+        resume = algo == "k_tm_walk"
+        blocks = work["resume_blocks_per_kernel" if resume else "run_blocks_per_kernel"] * (evals_step // n_f) / per_launch
         achieved = 32.0 * blocks / kern_avg_s / 1e9
         peak = 128.0 * sms * sm_max * 1e6 / 1e9
         roofline = {"bound": "l1", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                     "traffic": ncu_traffic(cfg) if args.models == "rf" else None, "kernel": algo,
                     "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "algorithmic_bytes_per_launch": 32.0 * blocks,
-                    "work": {"unit": "32-byte 2-level block fetches of the run walks", "per_launch": blocks,
+                    "work": {"unit": "32-byte 2-level block fetches of the " +
+                                     ("resume walks (each run restarts where its path leaves the previous run's)"
+                                      if resume else "run walks (each run restarts at the root)"),
+                             "per_launch": blocks,
                              "runs_per_kernel_tree": work["runs_per_kernel_tree"], "counted_on": work["sample"]},
                     "peak_note": f"L1/TEX load path 128 B/clk/SM x {sms} SMs x {sm_max:.0f} MHz (derived; "
                                  "not in MEASURED_PEAKS.json)",

@@ -72,13 +72,15 @@ int oracle_sweep(const oracle_model *speedup, const oracle_model *energy,
 
 /* oracle_sweep plus work counters of the run-walk algorithm (DESIGN.md §6 roofline): runs =
  * maximal clock runs sharing a leaf per (kernel, tree), run_decisions = sum of their leaf depths,
- * run_blocks = sum of max(1, ceil(depth/2)).  Counters are added to (not reset). */
+ * run_blocks = sum of max(1, ceil(depth/2)), resume_blocks = block fetches when every run after
+ * the first resumes at the block where its path leaves the previous run's (kernels_tm.cuh).
+ * Counters are added to (not reset). */
 int oracle_sweep_stats(const oracle_model *speedup, const oracle_model *energy,
                        const float *features, int64_t n_k, int32_t n_features,
                        const float *freqs, int32_t n_f, int32_t default_idx,
                        const int32_t *kind, const float *x, int32_t n_t,
                        int32_t *choice, int64_t *visits, int64_t *runs, int64_t *run_decisions,
-                       int64_t *run_blocks);
+                       int64_t *run_blocks, int64_t *resume_blocks);
 
 /* Four-model variant: models[0] speedup, [1] energy, [2] EDP, [3] ED2P
  * ([2]/[3] nullable = derived).  MIN_EDP / MIN_ED2P use the direct model's normalised

@@ -40,6 +40,7 @@ struct DevModel {
     // exact fixed-point leaf sums (k_sweep_da): every leaf v is an integer multiple of 2^-s and
     // n_trees * max|v| * 2^s < 2^62, so v * fx_scale is an exact int64 and sums are exact
     int fx_ok;
+    int fx32;                // fx_ok and every |v| * 2^s < 2^31 (int32 fixed-point leaves fit)
     double fx_scale;         // 2^s
     double fx_inv;           // 2^-s
     // SVR_RBF member: svr = b + sum_j dual_j exp(-gamma ||(x - mean)/scale - sv_j||^2)

@@ -1,0 +1,324 @@
+// kernels_tm.cuh — tree-major resume-walk sweep (k_tm_walk + k_tm_finish), the default fused path.
+//
+// What is computed is k_sweep_da's (kernels_da.cuh): per (kernel, model) the exact fixed-point sum
+// over trees of the leaf each clock reaches (Q8), accumulated as a difference array over
+// the clock axis, then the forest mean, linear / SVR members, default-clock normalisation and the
+// per-target masked argmin.  What changes is how the work is laid
+// on the machine, to cut L1 wavefronts, the resource k_sweep_da saturates (profiles/r1):
+//
+//  * Tree-major lanes.  A lane task is one (kernel, model, tree).  Tasks are numbered
+//      j = ((kernel block) * TT + tree) * KB + kernel-in-block
+//    and every CTA owns a contiguous range of j, so the lanes of an SM walk the SAME few trees for
+//    up to KB different kernels at once: the SM's L1 holds those trees, the 32 lanes of a warp
+//    load blocks of one tree (shared lines), and lines are reused by every kernel of the block.
+//    (k_sweep_da instead runs ~1000 different trees per SM and hits L1 9% of the time on c3.)
+//
+//  * Resume walks.  For a fixed kernel a tree is a step function of the clock index.  walk(lo)
+//    follows clock lo's path; the run is [lo, hi) with hi = #{i : f_i <= thr} minimised over the
+//    clock splits where the walk went LEFT.  The next clock hi follows the same path down to the
+//    first split that sends it right: the shallowest left-turn split whose cut equals hi (static
+//    splits do not depend on the clock, right turns stay right for a larger clock, and a left
+//    turn with a larger cut stays left).  So each lane keeps the prefix-minimum ("record") cuts
+//    of its path with their blocks, one entry per block, deepest on top: the next walk resumes at
+//    the top record's block (popped; the block is re-decided), and the new bound is the next
+//    record.  The stack keeps the kTmS deepest records; if it empties after shallower records
+//    were dropped, the walk restarts at the root.  On the bench forests this fetches 0.47x the
+//    blocks of root restarts.
+//
+//  * Clock cuts instead of clock values.  For a given clock table every clock-split threshold
+//    thr is replaced (k_cut_blocks, once per (model, clock table)) by its cut index
+//    c = #{i : f_i <= thr}, an integer exact in fp32, and clock i enters the walk as the value
+//    i + 0.5: f_i <= thr  <=>  i < c  <=>  i + 0.5 <= c, so every decision is unchanged.  The
+//    run end is then simply hi = min c over the left-turn clock splits (no search in the clock
+//    table), and split e is where clock hi turns right iff c_e < hi + 0.5.
+//
+//  * Step-level lockstep.  Every loop iteration is one 2-level block step for every busy lane; a
+//    lane that reaches a leaf closes its run and resumes in the same iteration, so walks of
+//    different lengths do not idle lanes.
+//
+//  * Accumulation in L2.  Run j of a (kernel, model, tree) adds v_j - v_{j-1} to
+//    D[kernel][slot][lo_j] with one 64-bit global reduction (exact, order-free; run 0 adds v_0).
+//    No shared-memory difference arrays: shared memory stays ~15 KB per CTA so L1 keeps the
+//    trees.  k_tm_finish then scans each D row (exact int64 prefix sum = the exact leaf sum per
+//    clock), rounds it once, combines the members and runs finish_tile4; it zeroes D as it reads
+//    it, so the next call starts from zeros without a memset.
+#pragma once
+#include "kernels_da.cuh"
+
+namespace syn {
+
+constexpr int kTmS = 4;          // resume-stack entries per lane (shallowest kept)
+constexpr int kTmNT = 512;       // k_tm_walk threads per CTA (2 CTAs per SM)
+
+struct TmArgs {
+    SweepArgs s;                 // models, clocks, targets, outputs of the whole call
+    long long* D;                // [nks][nslot][n_f] int64 difference arrays, zero on entry
+    long long slab0;             // global index of the slab's first kernel
+    long long n_tasks;           // ceil(nks / kb) * TT * kb lane tasks
+    int nks;                     // kernels in this slab
+    int kb;                      // kernels per feature block (power of two, 32..256)
+    int kb_log2;
+    int fx32;                    // every forest's leaves are int32 fixed-point in its cut blocks
+    int nslot;                   // D slots = models with a forest member
+    int slot_of[4];              // model -> D slot, -1 without forest
+    int nm;                      // models in the call (2 or 4)
+};
+
+template <int NT>
+__global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
+    const SweepArgs& a = t.s;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int n_f = a.n_f, F = a.F, KB = t.kb;
+    const int FR = max(F, 1);                                                // feature rows staged
+    int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
+    float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
+    float* xs = stk_c + kTmS * NT;                                           // [FR][KB] features
+    int* counter = reinterpret_cast<int*>(xs + (size_t)FR * KB);
+
+    const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
+              T3 = t.nm > 2 ? da_trees(a, 3) : 0;
+    const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
+    const long long per_kb = (long long)TT * KB;
+    const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
+    const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
+
+    const int lane = threadIdx.x & 31;
+    const unsigned lm_lt = lanemask_lt();
+    const unsigned xs_a = su32(xs);
+    const unsigned xstride = 4u * (unsigned)KB;
+    const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
+    constexpr unsigned kEnt = 4u * NT;                                       // bytes between entries
+    const int Fm1 = FR - 1;
+
+    for (long long s0 = r0; s0 < r1;) {
+        const long long kbi = s0 / per_kb;
+        const long long s1 = min(r1, (kbi + 1) * per_kb);
+        const int kbase = (int)(kbi * KB);                                   // slab-relative
+        __syncthreads();                                                     // previous block done
+        const float* gfeat = a.features + (t.slab0 + kbase) * F;
+        const int nvalid = min(KB, t.nks - kbase);
+        for (int e = threadIdx.x; e < KB * F; e += NT) {
+            const int kk = e / F, c = e - kk * F;
+            xs[c * KB + kk] = kk < nvalid ? __ldg(gfeat + e) : 0.0f;
+        }
+        if (threadIdx.x == 0) *counter = 0;
+        __syncthreads();
+
+        bool active = false, exhausted = false, lost = false;
+        const uint4* blocks = a.ms.blocks;
+        long long* drow = t.D;
+        double scale = 1.0;
+        unsigned xcol_a = xs_a;
+        int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
+        float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
+        long long vprev = 0;
+        while (true) {
+            // refill: idle lanes take the next lane tasks of this CTA's range (warp-aggregated)
+            const bool want = !active && !exhausted;
+            const unsigned need = __ballot_sync(0xffffffffu, want);
+            if (need) {
+                int base = 0;
+                const int leader = __ffs(need) - 1;
+                if (lane == leader) base = atomicAdd(counter, __popc(need));
+                base = __shfl_sync(0xffffffffu, base, leader);
+                if (want) {
+                    const long long j = s0 + base + __popc(need & lm_lt);
+                    if (j < s1) {
+                        const int rem = (int)(j - kbi * per_kb);
+                        const int tti = rem >> t.kb_log2, kk = rem & (KB - 1);
+                        if (kk < nvalid) {
+                            const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
+                            const int tree = tti - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3);
+                            const DevModel& m = da_model(a, mi);
+                            blocks = m.blocks;
+                            scale = m.fx_scale;
+                            root = __ldg(m.broot + tree);
+                            drow = t.D + ((kbase + kk) * t.nslot + t.slot_of[mi]) * n_f;
+                            xcol_a = xs_a + 4u * (unsigned)kk;
+                            bk = root;
+                            lo = 0;
+                            f_lo = 0.5f;
+                            tmin = CUDART_INF_F;
+                            sn = 0;
+                            lost = false;
+                            vprev = 0;
+                            active = true;
+                        }
+                    } else {
+                        exhausted = true;
+                    }
+                }
+            }
+            if (__all_sync(0xffffffffu, exhausted)) break;
+            if (active) {
+                // one 2-level block step (internal.h layout), branch-free; cb = smallest cut of
+                // this block's left-turn clock splits.  Static features are read at a clamped
+                // row whatever the code, then selected.
+                uint4 A, B;
+                const int cur = bk;
+                ldg_blk256(blocks + 2 * (size_t)cur, A, B);
+                const unsigned codes = A.w;
+                const int cn = (int)(codes & 0xffu);
+                const float xs_n = lds_f(xcol_a + xstride * (unsigned)min(cn, Fm1));
+                const float xn = cn == F ? f_lo : xs_n;
+                const bool l0 = xn <= __uint_as_float(A.x);
+                float cb = (cn == F && l0) ? __uint_as_float(A.x) : CUDART_INF_F;
+                const unsigned tcb = l0 ? A.y : A.z;
+                const int cc = (int)((codes >> (l0 ? 8 : 16)) & 0xffu);
+                const float xs_c = lds_f(xcol_a + xstride * (unsigned)min(cc, Fm1));
+                const float xc = cc == F ? f_lo : xs_c;
+                const bool l1 = xc <= __uint_as_float(tcb);
+                if (cc == F && l1) cb = fminf(cb, __uint_as_float(tcb));
+                const unsigned g = l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
+                const int slot = (l0 ? 0 : 2) + (l1 ? 0 : 1);
+                const bool leaf_n = cn > F, leaf_c = cc > F;
+                const bool at_leaf = leaf_n || leaf_c || ((codes >> (24 + slot)) & 1u);
+                const unsigned leafbits = leaf_n ? A.x : leaf_c ? tcb : g;   // one-leaf / child / grandchild
+                bk = (int)g;
+                if (cb < tmin) {                                             // new record: push
+                    sts_u(sb_a + kEnt * (unsigned)wp, (unsigned)cur);
+                    sts_f(sc_a + kEnt * (unsigned)wp, cb);
+                    wp = (wp + 1) & (kTmS - 1);
+                    lost = lost || sn == kTmS;
+                    sn = min(sn + 1, kTmS);
+                    tmin = cb;
+                }
+                if (at_leaf) {
+                    // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
+                    const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
+                    const long long v = t.fx32 ? (long long)(int)leafbits     // int32 fixed point
+                                               : __double2ll_rn(__dmul_rn((double)__uint_as_float(leafbits), scale));
+                    atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
+                    vprev = v;
+                    active = hi < n_f;
+                    // resume at the top record's block (popped); a stack emptied after dropping
+                    // shallower records restarts at the root
+                    wp = (wp + kTmS - 1) & (kTmS - 1);
+                    bk = (int)lds_u(sb_a + kEnt * (unsigned)wp);
+                    --sn;
+                    tmin = sn > 0 ? lds_f(sc_a + kEnt * (unsigned)((wp + kTmS - 1) & (kTmS - 1))) : CUDART_INF_F;
+                    if (sn == 0 && lost) {
+                        bk = root;
+                        lost = false;
+                    }
+                    lo = hi;
+                    f_lo = (float)hi + 0.5f;
+                }
+            }
+        }
+        s0 = s1;
+    }
+}
+
+// Clock-specialised copy of a model's 2-level blocks (see the header): every clock-split
+// threshold (code == F) becomes its cut index #{i : f_i <= thr} as an fp32 integer.  One thread
+// per block; child-leaf values (code F + 1) and grandchild slots are copied unchanged.
+__global__ void __launch_bounds__(256) k_cut_blocks(const uint4* __restrict__ in, long long n_blocks, int F,
+                                                    const float* __restrict__ freqs, int n_f,
+                                                    double fx_scale, uint4* __restrict__ out) {
+    const long long b = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (b >= n_blocks) return;
+    uint4 A = in[2 * b];
+    const uint4 B = in[2 * b + 1];
+    unsigned w[3] = {A.x, A.y, A.z};
+    unsigned g[4] = {B.x, B.y, B.z, B.w};
+#pragma unroll
+    for (int q = 0; q < 3; ++q) {
+        const int code = (int)((A.w >> (8 * q)) & 0xffu);
+        if (code > F && fx_scale != 0.0) {
+            // leaf value (one-leaf tree at q = 0, child leaf at q = 1, 2) -> int32 v * 2^s, exact
+            w[q] = (unsigned)__double2int_rn(__dmul_rn((double)__uint_as_float(w[q]), fx_scale));
+            continue;
+        }
+        if (code != F) continue;
+        const float thr = __uint_as_float(w[q]);
+        int l = 0, h = n_f;                                  // #{i : f_i <= thr}
+        while (l < h) {
+            const int mid = (l + h) >> 1;
+            if (__ldg(freqs + mid) <= thr) l = mid + 1; else h = mid;
+        }
+        w[q] = __float_as_uint((float)l);
+    }
+    if (fx_scale != 0.0) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if ((A.w >> (24 + q)) & 1u) g[q] = (unsigned)__double2int_rn(__dmul_rn((double)__uint_as_float(g[q]), fx_scale));
+    }
+    A.x = w[0];
+    A.y = w[1];
+    A.z = w[2];
+    out[2 * b] = A;
+    out[2 * b + 1] = make_uint4(g[0], g[1], g[2], g[3]);
+}
+
+// Finish of KT kernels per CTA: exact prefix sums of the D rows (zeroing them), forest mean,
+// linear member, then finish_tile4 (SVR members, normalisation, selection).
+__global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArgs t) {
+    const SweepArgs& a = t.s;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int n_f = a.n_f, F = a.F, KT = a.tile_k, XS = a.xs, NM = t.nm;
+    const int k0s = blockIdx.x * KT;
+    const int nk = min(KT, t.nks - k0s);
+    const long long k0 = t.slab0 + k0s;
+    double* mv0 = reinterpret_cast<double*>(smem);                            // [NM][KT][n_f]
+    float* sv0 = reinterpret_cast<float*>(mv0 + (size_t)NM * KT * n_f);       // [NM][KT][n_f]
+    float* fr = sv0 + (size_t)NM * KT * n_f;
+    float* xk = fr + n_f;                                                     // [KT][XS]
+    long long* sD = reinterpret_cast<long long*>(xk + KT * XS + 1);           // [KT][nslot][n_f]
+    sD = reinterpret_cast<long long*>((reinterpret_cast<uintptr_t>(sD) + 15) & ~(uintptr_t)15);
+    const float* gfeat = a.features + k0 * F;
+    for (int e = threadIdx.x; e < nk * F; e += blockDim.x) {
+        const int r = e / F;
+        xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
+    }
+    for (int i = threadIdx.x; i < n_f; i += blockDim.x) fr[i] = __ldg(a.freqs + i);
+    // this CTA's D rows are one contiguous region: stage it with independent coalesced loads,
+    // then zero it for the next call
+    long long* gD = t.D + (size_t)k0s * t.nslot * n_f;
+    const int nd = nk * t.nslot * n_f;
+    for (int e = threadIdx.x; e < nd; e += blockDim.x) sD[e] = __ldcg(gD + e);
+    __syncthreads();
+    for (int e = threadIdx.x; e < nd; e += blockDim.x) gD[e] = 0;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    for (int p = warp; p < NM * nk; p += nw) {                                // p = kernel * NM + model
+        const int pk = p / NM, pm = p - pk * NM;
+        if (pm >= 2 && !a.has_x[pm - 2]) continue;
+        const DevModel& m = da_model(a, pm);
+        double* out = mv0 + ((size_t)pm * KT + pk) * n_f;
+        const float* xrow = xk + pk * XS;
+        const int slot = t.slot_of[pm];
+        if (slot < 0) {
+            for (int i = lane; i < n_f; i += 32) out[i] = combine(m, 0.0, xrow, fr[i], F);
+            continue;
+        }
+        const long long* Dm = sD + ((size_t)pk * t.nslot + slot) * n_f;
+        const int chunk = (n_f + 31) / 32;
+        const int i0 = min(n_f, lane * chunk), i1 = min(n_f, i0 + chunk);
+        long long run = 0;
+        for (int i = i0; i < i1; ++i) run += Dm[i];
+        long long excl = run;                                                 // inclusive scan of chunk sums
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const long long y = __shfl_up_sync(0xffffffffu, excl, off);
+            if (lane >= off) excl += y;
+        }
+        excl -= run;
+        const double inv = m.fx_inv;
+        for (int i = i0; i < i1; ++i) {
+            excl += Dm[i];
+            const double forest_sum = __dmul_rn(__ll2double_rn(excl), inv);  // RN(exact sum)
+            out[i] = combine(m, forest_sum, xrow, fr[i], F);
+        }
+    }
+    __syncthreads();
+    double* mv[4];
+    float* sv[4];
+    for (int m = 0; m < 4; ++m) {
+        const bool present = m < 2 || (NM > 2 && a.has_x[m - 2]);
+        mv[m] = present ? mv0 + (size_t)m * KT * n_f : nullptr;
+        sv[m] = present ? sv0 + (size_t)m * KT * n_f : nullptr;
+    }
+    finish_tile4(a, mv, sv, nk, k0);
+}
+
+}  // namespace syn

@@ -3,11 +3,13 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <list>
 #include <mutex>
 #include <new>
 #include <string>
@@ -19,6 +21,7 @@
 #include "kernels_ws.cuh"
 #include "kernels_da.cuh"
 #include "kernels_svr.cuh"
+#include "kernels_tm.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -32,6 +35,8 @@ struct syn_model {
     long long bytes;
     void* alloc;
     DevModel dm;
+    long long n_blocks;                                   // 2-level blocks (2 x uint4 each)
+    std::vector<std::pair<long long, uint4*>> cut_blocks;  // per clock table (uid): k_cut_blocks copy
 };
 
 struct syn_clocks {
@@ -40,6 +45,7 @@ struct syn_clocks {
     float* d_freqs;
     unsigned short* d_grid;   // clock-cut hint table, kGrid + 1 entries
     float f0, inv_step;
+    long long uid;            // unique per created table (keys the models' clock-cut block copies)
 };
 
 struct syn_workspace {
@@ -374,6 +380,200 @@ cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaS
     return topc ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
 }
 
+// ------------------------------------------------------------------ tree-major path (kernels_tm.cuh)
+// D difference arrays live in a library-owned buffer per (device, stream).  k_tm_finish zeroes
+// every entry it reads, so a buffer is all-zero between calls on its stream; a call that fails
+// after enqueuing k_tm_walk marks it dirty and the next call clears it with a memset.
+struct TmBuf {
+    int dev;
+    cudaStream_t st;
+    long long* p;
+    size_t bytes;
+    bool dirty;
+};
+std::mutex g_tm_mu;
+std::list<TmBuf> g_tm_bufs;          // list: entries never move
+
+syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out) {
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    TmBuf* b = nullptr;
+    for (TmBuf& x : g_tm_bufs)
+        if (x.dev == dev && x.st == st) b = &x;
+    if (!b) {
+        g_tm_bufs.push_back({dev, st, nullptr, 0, false});
+        b = &g_tm_bufs.back();
+    }
+    cudaError_t e = cudaSuccess;
+    if (b->bytes < bytes) {
+        if (b->p) {
+            cudaStreamSynchronize(st);          // the old buffer may still be read by queued work
+            cudaFree(b->p);
+            b->p = nullptr;
+            b->bytes = 0;
+        }
+        if ((e = cudaMalloc(&b->p, bytes)) != cudaSuccess) {
+            cudaGetLastError();
+            b->p = nullptr;
+            return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "tree-major D buffer of %zu bytes", bytes)
+                                                  : cuda_fail(e, "cudaMalloc(D)");
+        }
+        b->bytes = bytes;
+        b->dirty = true;
+    }
+    if (b->dirty) {
+        if ((e = cudaMemsetAsync(b->p, 0, b->bytes, st)) != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(D)");
+        b->dirty = false;
+    }
+    *out = b;
+    return ok();
+}
+
+// Clock-cut copy of a model's blocks for one clock table (kernels_tm.cuh, k_cut_blocks), built on
+// first use and cached in the model.  The build is synchronous (once per model and table) so any
+// stream may use the copy afterwards.
+std::mutex g_cut_mu;
+syn_status cut_blocks(syn_model* m, const syn_clocks* c, const uint4** out) {
+    std::lock_guard<std::mutex> lock(g_cut_mu);
+    for (auto& cb : m->cut_blocks)
+        if (cb.first == c->uid) {
+            *out = cb.second;
+            return ok();
+        }
+    uint4* p = nullptr;
+    const long long nb = std::max<long long>(m->n_blocks, 1);
+    cudaError_t e = cudaMalloc(&p, (size_t)nb * 2 * sizeof(uint4));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return cuda_fail(e, "cudaMalloc(clock-cut blocks)");
+    }
+    if (m->n_blocks > 0)
+        k_cut_blocks<<<(unsigned)((m->n_blocks + 255) / 256), 256>>>(m->dm.blocks, m->n_blocks, m->n_inputs - 1,
+                                                                   c->d_freqs, c->n_f, m->dm.fx32 ? m->dm.fx_scale : 0.0, p);
+    if ((e = cudaGetLastError()) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess) {
+        cudaFree(p);
+        return cuda_fail(e, "k_cut_blocks");
+    }
+    m->cut_blocks.push_back({c->uid, p});
+    *out = p;
+    return ok();
+}
+
+constexpr size_t kTmSlabBytes = 48u << 20;   // D bytes per slab (stays L2-resident with the model)
+
+// Tree-major path (k_tm_walk + k_tm_finish per kernel slab).  Needs every forest within the exact
+// int64 leaf range (fx_ok) and at least one tree; returns false (nothing enqueued) otherwise.
+bool tm_eligible(const SweepArgs& a, int nm) {
+    int tt = 0;
+    for (int m = 0; m < nm; ++m) {
+        if (m >= 2 && !a.has_x[m - 2]) continue;
+        const DevModel& d = m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+        if (d.forest_weight == 0.0 || d.n_trees == 0) continue;
+        if (!d.fx_ok) return false;
+        tt += d.n_trees;
+    }
+    return tt > 0;
+}
+
+syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clocks* clocks, cudaStream_t st,
+                  int* launches) {
+    const int device = clocks->device;
+    DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
+    for (int m = 0; m < nm; ++m) {
+        if (!models[m] || dms[m]->forest_weight == 0.0 || dms[m]->n_trees == 0) continue;
+        const uint4* cb = nullptr;
+        syn_status cs = cut_blocks(models[m], clocks, &cb);
+        if (cs != SYN_OK) return cs;
+        dms[m]->blocks = cb;
+    }
+    TmArgs t;
+    memset(&t, 0, sizeof t);
+    const int n_f = a.n_f, F = a.F;
+    const long long n_k = a.n_k;
+    int tt = 0;
+    t.nslot = 0;
+    for (int m = 0; m < 4; ++m) {
+        t.slot_of[m] = -1;
+        if (m >= nm || (m >= 2 && !a.has_x[m - 2])) continue;
+        const DevModel& d = m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+        if (d.forest_weight == 0.0 || d.n_trees == 0) continue;
+        t.slot_of[m] = t.nslot++;
+        tt += d.n_trees;
+    }
+    t.nm = nm;
+    t.fx32 = 1;
+    for (int m = 0; m < nm; ++m)
+        if (t.slot_of[m] >= 0 && !dms[m]->fx32) t.fx32 = 0;
+    // kernels per feature block: a power of two in [32, 256], F * kb floats of shared memory
+    int kb = 256;
+    while (kb > 32 && ((size_t)F * kb * 4 > 32768 || kb / 2 >= n_k)) kb /= 2;
+    const int kb_env = env_int("SYNERGY_TM_KB", kb);
+    while (kb > 32 && kb > kb_env) kb /= 2;
+    while (kb < 256 && kb * 2 <= kb_env) kb *= 2;
+    t.kb = kb;
+    t.kb_log2 = 0;
+    while ((1 << t.kb_log2) < kb) ++t.kb_log2;
+    const size_t row = (size_t)t.nslot * n_f * sizeof(long long);
+    long long nks = std::max<long long>(kb, (long long)(kTmSlabBytes / row) / kb * kb);
+    nks = std::max<long long>(kb, env_int("SYNERGY_TM_SLAB", (int)std::min<long long>(nks, 1 << 30)) / kb * kb);
+    nks = std::min<long long>(nks, n_k);
+    TmBuf* buf = nullptr;
+    syn_status s = tm_buffer(device, st, (size_t)nks * row, &buf);
+    if (s != SYN_OK) return s;
+    t.D = buf->p;
+    // finish tile: KT kernels per CTA, fp64 + fp32 per (model, kernel, clock) in shared memory
+    // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
+    int kt = std::max(1, std::min(8, (int)((150 * 1024) / ((size_t)nm * n_f * 12 + (size_t)t.nslot * n_f * 8))));
+    kt = (int)std::max<long long>(1, std::min<long long>(kt, nks / (8LL * sm_count(device))));
+    kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
+    a.tile_k = kt;
+    a.xs = (F + 2) | 1;
+    const size_t fsmem = (size_t)nm * kt * n_f * 12 + (size_t)n_f * 4 + (size_t)kt * a.xs * 4 + 32 +
+                         (size_t)kt * t.nslot * n_f * 8;
+    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)std::max(F, 1) * kb * 4 + 16;
+    static size_t fset = 48 * 1024, wset = 48 * 1024;
+    cudaError_t e = cudaSuccess;
+    if (fsmem > fset) {
+        if ((e = cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem)) != cudaSuccess)
+            return cuda_fail(e, "k_tm_finish attribute");
+        fset = fsmem;
+    }
+    if (wsmem > wset) {
+        if ((e = cudaFuncSetAttribute(k_tm_walk<kTmNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess)
+            return cuda_fail(e, "k_tm_walk attribute");
+        wset = wsmem;
+    }
+    const int ctas = std::max(1, env_int("SYNERGY_TM_CTAS", 2 * sm_count(device)));
+    t.s = a;
+    int n = 0;
+    for (long long s0 = 0; s0 < n_k; s0 += nks) {
+        t.slab0 = s0;
+        t.nks = (int)std::min<long long>(nks, n_k - s0);
+        t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * kb;
+        const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
+        {
+            KernelTimer ktm("k_tm_walk", st);
+            k_tm_walk<kTmNT><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) {
+            buf->dirty = true;
+            return cuda_fail(e, "k_tm_walk launch");
+        }
+        {
+            KernelTimer ktm("k_tm_finish", st);
+            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), 256, fsmem, st>>>(t);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) {
+            buf->dirty = true;
+            return cuda_fail(e, "k_tm_finish launch");
+        }
+        n += 2;
+    }
+    *launches = n;
+    return ok();
+}
+
 template <int S, int T>
 cudaError_t launch_sweep_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
     static size_t smem_set = 48 * 1024;   // per-instantiation opt-in high-water mark
@@ -643,6 +843,16 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     syn_status ss = prepare_svr(a.ms, clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss == SYN_OK) ss = prepare_svr(a.me, clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss != SYN_OK) return ss;
+    // default: tree-major resume walks (kernels_tm.cuh) whenever the exact int64 leaf sums apply;
+    // SYNERGY_ALGO=da|ws|iv|direct selects one of the single-launch kernels instead
+    if (!algo_env && tm_eligible(a, 2)) {
+        int nl = 0;
+        syn_model* ms[2] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en)};
+        ss = run_tm(a, 2, ms, clocks, st, &nl);
+        if (ss != SYN_OK) return ss;
+        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k), kTmNT, 4000};
+        return ok();
+    }
     static const char* knames[4] = {"k_sweep", "k_sweep_iv", "k_sweep_ws", "k_sweep_da"};
     cudaError_t e;
     {
@@ -752,7 +962,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         }
     }
     // exact fixed-point scale for the leaf sums (k_sweep_da): s = -(smallest leaf ulp exponent)
-    int fx_ok = 0, fx_s = 0;
+    int fx_ok = 0, fx_s = 0, fx32 = 0;
     if (d->forest_weight != 0.0) {
         int min_lsb = 1 << 30, max_e = -(1 << 30);
         bool finite = true;
@@ -768,12 +978,13 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
                 max_e = std::max(max_e, e2);
             }
         if (finite) {
-            if (max_e == -(1 << 30)) { fx_ok = 1; fx_s = 0; }   // all leaves zero
+            if (max_e == -(1 << 30)) { fx_ok = 1; fx_s = 0; fx32 = 1; }   // all leaves zero
             else {
                 fx_s = -min_lsb;
                 int lg = 0;
                 while ((1LL << lg) < (long long)d->n_trees + 1) ++lg;
                 fx_ok = (max_e + fx_s + lg <= 61) ? 1 : 0;
+                fx32 = (fx_ok && max_e + fx_s <= 31) ? 1 : 0;
             }
         }
     }
@@ -894,7 +1105,9 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
     m->dm.bdepth = bdepth;
+    m->n_blocks = (long long)(blocks.size() >> 1);
     m->dm.fx_ok = fx_ok;
+    m->dm.fx32 = fx32;
     m->dm.fx_scale = std::ldexp(1.0, fx_s);
     m->dm.fx_inv = std::ldexp(1.0, -fx_s);
     m->dm.svr_weight = d->svr_weight;
@@ -918,6 +1131,7 @@ syn_status synergy_model_destroy(syn_model* m) {
     {
         DeviceGuard g(m->device);
         cudaFree(m->alloc);
+        for (auto& cb : m->cut_blocks) cudaFree(cb.second);
     }
     delete m;
     return ok();
@@ -975,6 +1189,8 @@ syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, sy
     c->d_grid = reinterpret_cast<unsigned short*>(reinterpret_cast<char*>(d) + goff);
     c->f0 = f0;
     c->inv_step = 1.0f / step;
+    static std::atomic<long long> next_uid{1};
+    c->uid = next_uid++;
     *out = c;
     return ok();
 }
@@ -1076,6 +1292,16 @@ syn_status synergy_sweep4(const syn_model* const* models, const float* d_feature
     for (int m = 0; m < 4 && ss == SYN_OK; ++m)
         if (m < 2 || a.has_x[m - 2]) ss = prepare_svr(*dms[m], clocks->device, d_features, n_k, F, clocks, st, scr);
     if (ss != SYN_OK) return ss;
+    const char* algo_env = getenv("SYNERGY_ALGO");
+    if (!algo_env && tm_eligible(a, 4)) {
+        int nl = 0;
+        syn_model* ms[4] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en), const_cast<syn_model*>(x2),
+                            const_cast<syn_model*>(x3)};
+        ss = run_tm(a, 4, ms, clocks, st, &nl);
+        if (ss != SYN_OK) return ss;
+        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k), kTmNT, 4000};
+        return ok();
+    }
     cudaError_t e;
     {
         KernelTimer kt("k_sweep_da", st);

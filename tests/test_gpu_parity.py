@@ -22,7 +22,11 @@ def _build():
 
 
 # Kernel variants the library can pick (read per call from the environment):
-#   default   order-free difference-array kernel (k_sweep_da), exact int64 leaf sums
+#   default   tree-major resume walks (k_tm_walk + k_tm_finish), exact int64 leaf sums in L2
+#   tm_kb32   k_tm_walk with 32-kernel feature blocks (several blocks per CTA range)
+#   tm_ctas3  k_tm_walk on 3 CTAs (long per-CTA ranges crossing kernel blocks, many tasks/lane)
+#   tm_slab   kernel slabs of 64 (several walk + finish launches reusing the zeroed D buffer)
+#   da        order-free difference-array kernel (k_sweep_da), shared-memory int64 sums
 #   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
 #   da_nt256  k_sweep_da with 256 threads per CTA
 #   da_kpc5   k_sweep_da with 5 kernels per CTA (tasks of several kernels per warp, ragged tile)
@@ -38,8 +42,13 @@ def _build():
 #   iv_vcap1  k_sweep_iv keeping 1 run value per (kernel, tree)
 #   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
-VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERGY_NT": "256"},
-            "da_kpc5": {"SYNERGY_KPC": "5"}, "da_nsub3": {"SYNERGY_NSUB": "3"}, "da_nsub64": {"SYNERGY_NSUB": "64", "SYNERGY_KPC": "2"}, "da_topc": {"SYNERGY_TOPC": "1", "SYNERGY_KPC": "3"},
+DA = {"SYNERGY_ALGO": "da"}
+VARIANTS = {"default": {}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
+            "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
+            "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
+            "da_kpc5": {**DA, "SYNERGY_KPC": "5"}, "da_nsub3": {**DA, "SYNERGY_NSUB": "3"},
+            "da_nsub64": {**DA, "SYNERGY_NSUB": "64", "SYNERGY_KPC": "2"},
+            "da_topc": {**DA, "SYNERGY_TOPC": "1", "SYNERGY_KPC": "3"},
             "ws": {"SYNERGY_ALGO": "ws"},
             "ws_tight": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"},
             "ws_wide": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
@@ -47,7 +56,7 @@ VARIANTS = {"default": {}, "da_nt64": {"SYNERGY_NT": "64"}, "da_nt256": {"SYNERG
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+KNOBS = ("SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
@@ -97,6 +106,9 @@ FUZZ = [
     (300, 128, 12, 3, 6, "none", {}),
     (1100, 40, 6, 2, 4, "none", {"value_range": (-0.5, 1.5)}),        # non-positive predictions
     (40, 50, 6, 2, 0, "none", {}),                                    # depth-0 stumps: constant
+    (23, 196, 4, 5, 14, "none", {"p_freq": 0.9, "p_leaf": 0.05}),    # clock-heavy: resume stack overflows
+    (29, 64, 3, 4, 16, "none", {"p_freq": 0.7, "p_leaf": 0.02, "exact_thresholds": True}),
+    (600, 64, 5, 4, 9, "both", {"p_freq": 0.5}),                      # 3 kernel blocks, ragged last
 ]
 
 
@@ -140,7 +152,7 @@ def test_exact_sum_where_sequential_fp64_rounds():
     w = _stump_models(vals, [1.0, 2.0])
     S, E = gpu_predict(w, default_idx=-1)
     rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
-    assert syn.last_launch()["variant"] // 1000 == 3          # difference-array kernel ran
+    assert syn.last_launch()["variant"] // 1000 in (3, 4)     # an exact int64 kernel ran
     assert_bits_equal(S, rS, "raw S")
     assert_bits_equal(E, rE, "raw E")
 
@@ -152,7 +164,7 @@ def test_out_of_range_leaves_fall_back_to_ordered_kernel():
     w = _stump_models([2.0 ** 60, 2.0 ** -60], [1.0, 0.5])
     S, E = gpu_predict(w, default_idx=-1)
     rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
-    assert syn.last_launch()["variant"] // 1000 != 3
+    assert syn.last_launch()["variant"] // 1000 not in (3, 4)
     assert_bits_equal(S, rS, "raw S")
     assert_bits_equal(E, rE, "raw E")
 
@@ -172,8 +184,8 @@ def _gpu_sweep4(models, feats, freqs, d, targets):
 @pytest.mark.parametrize("cfg", ["c1", "c2"])
 def test_four_model_variant_bit_exact(cfg, variant):
     """NEXT f1: speedup + energy + direct EDP (RF) + direct ED2P (linear)."""
-    if VARIANTS[variant].get("SYNERGY_ALGO"):
-        pytest.skip("four-model sweep always runs on k_sweep_da")
+    if VARIANTS[variant].get("SYNERGY_ALGO", "da") != "da":
+        pytest.skip("four-model sweep runs on the exact int64 kernels only")
     models, freqs, d = W.make_models4(cfg)
     feats = W.make_features(cfg)
     targets = W.targets_six()

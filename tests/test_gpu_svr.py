@@ -54,7 +54,7 @@ def env(request):
             os.environ[k] = v
 
 
-ALGOS = ["", "ws", "iv", "direct"]
+ALGOS = ["", "da", "ws", "iv", "direct"]
 
 
 @pytest.mark.parametrize("ensemble", [False, True])
@@ -67,7 +67,8 @@ def test_svr_sweep_matches_oracle(env, ensemble, algo, splits):
     ref = oracle.sweep(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets, want_pred=True)
     got = gpu_sweep(w, want_pred=True)
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
-    assert syn.last_launch()["kernels"] == 4     # k_svr_v + k_svr_u + k_svr + the sweep kernel
+    # k_svr_v + k_svr_u + k_svr + the sweep (tree-major default: walk + finish)
+    assert syn.last_launch()["kernels"] == (5 if algo == "" else 4)
     check_pred(got["S"], ref["S"], "S")
     dE = check_pred(got["E"], ref["E"], "E")
     np.testing.assert_array_equal(got["choice"], oracle.select(got["S"], got["E"], w.default_idx, w.targets))

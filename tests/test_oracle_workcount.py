@@ -8,14 +8,20 @@ from paper_conf_sc_fandccfc23_b200 import workloads as W
 
 
 def interval_runs(spec, t, x_static, freqs):
-    """(runs, sum of leaf depths, sum of max(1, ceil(depth/2))) for one (kernel, tree)."""
+    """(runs, sum of leaf depths, sum of max(1, ceil(depth/2)), resume-walk block fetches) for one
+    (kernel, tree).  Resume fetches, counted per reachable node: every 2-level block (the root and
+    every reachable internal node at even depth) is fetched once when first reached, plus once
+    more for every clock split inside it (its node or the reachable child) whose reachable clock
+    interval has clocks on both sides: the first clock of the right side resumes at that block."""
     base = spec.tree_offset[t]
     F = len(x_static)
-    runs = dec = blk = 0
+    runs = dec = blk = res = 0
     stack = [(0, 0, len(freqs), 0)]
     while stack:
         n, lo, hi, d = stack.pop()
         f = spec.feature[base + n]
+        if d % 2 == 0 and (f >= 0 or d == 0):
+            res += 1                                           # block first reached
         if f < 0:
             runs += 1
             dec += d
@@ -27,27 +33,31 @@ def interval_runs(spec, t, x_static, freqs):
             stack.append((L if x_static[f] <= thr else R, lo, hi, d + 1))
             continue
         s = int(np.searchsorted(freqs, thr, side="right"))     # #clocks <= thr
+        if lo < s < hi:
+            res += 1                                           # right side resumes at this block
         if s < hi and max(s, lo) < hi:
             stack.append((R, max(s, lo), hi, d + 1))
         if s > lo:
             stack.append((L, lo, min(s, hi), d + 1))
-    return runs, dec, blk
+    return runs, dec, blk, res
 
 
 def _check(w):
     import oracle
     r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
-    runs = dec = blk = 0
+    runs = dec = blk = res = 0
     for k in range(w.n_kernels):
         for m in (w.speedup, w.energy):
             if m.forest_weight == 0.0:
                 continue
             for t in range(m.n_trees):
-                a, b, c = interval_runs(m, t, w.features[k], w.freqs)
+                a, b, c, e = interval_runs(m, t, w.features[k], w.freqs)
                 runs += a
                 dec += b
                 blk += c
+                res += e
     assert (r["runs"], r["run_decisions"], r["run_blocks"]) == (runs, dec, blk)
+    assert r["resume_blocks"] == res
     np.testing.assert_array_equal(r["choice"], oracle.sweep_workload(w)["choice"])
 
 
