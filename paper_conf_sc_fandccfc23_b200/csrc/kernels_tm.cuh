@@ -73,17 +73,20 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
     float* xs = stk_c + kTmS * NT;                                           // [FR][KB] features
-    int* counter = reinterpret_cast<int*>(xs + (size_t)FR * KB);
+    int* sroot = reinterpret_cast<int*>(xs + (size_t)FR * KB);              // [TT] root block per tree
 
     const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
               T3 = t.nm > 2 ? da_trees(a, 3) : 0;
     const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
     const long long per_kb = (long long)TT * KB;
+    for (int q = threadIdx.x; q < TT; q += NT) {
+        const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
+        sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
+    }
     const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
     const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
 
     const int lane = threadIdx.x & 31;
-    const unsigned lm_lt = lanemask_lt();
     const unsigned xs_a = su32(xs);
     const unsigned xstride = 4u * (unsigned)KB;
     const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
@@ -101,7 +104,6 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             const int kk = e / F, c = e - kk * F;
             xs[c * KB + kk] = kk < nvalid ? __ldg(gfeat + e) : 0.0f;
         }
-        if (threadIdx.x == 0) *counter = 0;
         __syncthreads();
 
         bool active = false, exhausted = false, lost = false;
@@ -112,42 +114,45 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
         float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
         long long vprev = 0;
+        // Static lane streams: task j belongs to lane j % 32 and warp (j / 32) % NW, so a lane's
+        // kernel-in-block kk = j % KB is always = lane (mod 32) and its feature reads hit its own
+        // bank (no conflicts, no shared counter); consecutive 32-task groups (one tree, 32
+        // kernels) go to consecutive warps.
+        const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);   // segment offsets
+        int q;                                                                // this lane's next offset
+        {
+            const int nw = NT / 32, w = threadIdx.x >> 5;
+            const int g0 = seg0 >> 5;
+            int g = g0 + ((w - g0 % nw) + nw) % nw;
+            q = 32 * g + lane;
+            if (q < seg0) q += 32 * nw;
+        }
+        const int qstep = NT;                                                 // 32 * NW
         while (true) {
-            // refill: idle lanes take the next lane tasks of this CTA's range (warp-aggregated)
-            const bool want = !active && !exhausted;
-            const unsigned need = __ballot_sync(0xffffffffu, want);
-            if (need) {
-                int base = 0;
-                const int leader = __ffs(need) - 1;
-                if (lane == leader) base = atomicAdd(counter, __popc(need));
-                base = __shfl_sync(0xffffffffu, base, leader);
-                if (want) {
-                    const long long j = s0 + base + __popc(need & lm_lt);
-                    if (j < s1) {
-                        const int rem = (int)(j - kbi * per_kb);
-                        const int tti = rem >> t.kb_log2, kk = rem & (KB - 1);
-                        if (kk < nvalid) {
-                            const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
-                            const int tree = tti - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3);
-                            const DevModel& m = da_model(a, mi);
-                            blocks = m.blocks;
-                            scale = m.fx_scale;
-                            root = __ldg(m.broot + tree);
-                            drow = t.D + ((kbase + kk) * t.nslot + t.slot_of[mi]) * n_f;
-                            xcol_a = xs_a + 4u * (unsigned)kk;
-                            bk = root;
-                            lo = 0;
-                            f_lo = 0.5f;
-                            tmin = CUDART_INF_F;
-                            sn = 0;
-                            lost = false;
-                            vprev = 0;
-                            active = true;
-                        }
-                    } else {
-                        exhausted = true;
-                    }
+            if (!active && !exhausted) {
+                // refill: this lane's next task of the segment
+                while (q < seg1) {
+                    const int tti = q >> t.kb_log2, kk = q & (KB - 1);
+                    q += qstep;
+                    if (kk >= nvalid) continue;
+                    const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
+                    const DevModel& m = da_model(a, mi);
+                    blocks = m.blocks;
+                    scale = m.fx_scale;
+                    root = sroot[tti];
+                    drow = t.D + ((kbase + kk) * t.nslot + t.slot_of[mi]) * n_f;
+                    xcol_a = xs_a + 4u * (unsigned)kk;
+                    bk = root;
+                    lo = 0;
+                    f_lo = 0.5f;
+                    tmin = CUDART_INF_F;
+                    sn = 0;
+                    lost = false;
+                    vprev = 0;
+                    active = true;
+                    break;
                 }
+                if (!active) exhausted = true;
             }
             if (__all_sync(0xffffffffu, exhausted)) break;
             if (active) {

@@ -529,7 +529,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     a.xs = (F + 2) | 1;
     const size_t fsmem = (size_t)nm * kt * n_f * 12 + (size_t)n_f * 4 + (size_t)kt * a.xs * 4 + 32 +
                          (size_t)kt * t.nslot * n_f * 8;
-    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)std::max(F, 1) * kb * 4 + 16;
+    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)std::max(F, 1) * kb * 4 + 16 + (size_t)tt * 4;
     static size_t fset = 48 * 1024, wset = 48 * 1024;
     cudaError_t e = cudaSuccess;
     if (fsmem > fset) {
