@@ -59,6 +59,9 @@ struct TmArgs {
     int kb;                      // kernels per feature block (power of two, 32..256)
     int kb_log2;
     int fx32;                    // every forest's leaves are int32 fixed-point in its cut blocks
+    int ilv;                     // interleaved mode (small slabs): all slab features staged, CTA c
+                                 // takes chunks c, c + G, ... of (tree, 32-kernel group)
+    int ng;                      // 32-kernel groups in the slab (ilv)
     int nslot;                   // D slots = models with a forest member
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
@@ -83,8 +86,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
         sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
     }
-    const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
-    const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
+    const long long r0 = t.ilv ? 0 : (long long)blockIdx.x * t.n_tasks / gridDim.x;
+    const long long r1 = t.ilv ? 1 : (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
 
     const int lane = threadIdx.x & 31;
     const unsigned xs_a = su32(xs);
@@ -94,12 +97,12 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     const int Fm1 = FR - 1;
 
     for (long long s0 = r0; s0 < r1;) {
-        const long long kbi = s0 / per_kb;
-        const long long s1 = min(r1, (kbi + 1) * per_kb);
+        const long long kbi = t.ilv ? 0 : s0 / per_kb;
+        const long long s1 = t.ilv ? r1 : min(r1, (kbi + 1) * per_kb);
         const int kbase = (int)(kbi * KB);                                   // slab-relative
         __syncthreads();                                                     // previous block done
         const float* gfeat = a.features + (t.slab0 + kbase) * F;
-        const int nvalid = min(KB, t.nks - kbase);
+        const int nvalid = min(KB, t.nks - kbase);                           // (ilv: KB = 32 * ng)
         for (int e = threadIdx.x; e < KB * F; e += NT) {
             const int kk = e / F, c = e - kk * F;
             xs[c * KB + kk] = kk < nvalid ? __ldg(gfeat + e) : 0.0f;
@@ -118,21 +121,35 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         // kernel-in-block kk = j % KB is always = lane (mod 32) and its feature reads hit its own
         // bank (no conflicts, no shared counter); consecutive 32-task groups (one tree, 32
         // kernels) go to consecutive warps.
-        const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);   // segment offsets
+        // Interleaved mode: chunk ch = (tree ch / ng, kernel group ch % ng) of 32 tasks; CTA c's
+        // warp w takes chunks c + G * (w + NW * m), lane L its kernel 32 * group + L.
+        const int seg0 = (int)(s0 - kbi * per_kb), seg1 = t.ilv ? TT * t.ng : (int)(s1 - kbi * per_kb);
         int q;                                                                // this lane's next offset
+        int qstep = NT;                                                       // 32 * NW
         {
             const int nw = NT / 32, w = threadIdx.x >> 5;
-            const int g0 = seg0 >> 5;
-            int g = g0 + ((w - g0 % nw) + nw) % nw;
-            q = 32 * g + lane;
-            if (q < seg0) q += 32 * nw;
+            if (t.ilv) {
+                q = blockIdx.x + gridDim.x * w;                               // chunk index
+                qstep = gridDim.x * nw;
+            } else {
+                const int g0 = seg0 >> 5;
+                int g = g0 + ((w - g0 % nw) + nw) % nw;
+                q = 32 * g + lane;
+                if (q < seg0) q += 32 * nw;
+            }
         }
-        const int qstep = NT;                                                 // 32 * NW
         while (true) {
             if (!active && !exhausted) {
                 // refill: this lane's next task of the segment
                 while (q < seg1) {
-                    const int tti = q >> t.kb_log2, kk = q & (KB - 1);
+                    int tti, kk;
+                    if (t.ilv) {
+                        tti = q / t.ng;
+                        kk = 32 * (q - tti * t.ng) + lane;
+                    } else {
+                        tti = q >> t.kb_log2;
+                        kk = q & (KB - 1);
+                    }
                     q += qstep;
                     if (kk >= nvalid) continue;
                     const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
