@@ -91,11 +91,14 @@ def load_peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
-def ncu_traffic(cfg):
+def ncu_traffic(cfg, kernel="k_sweep_da"):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of `kernel` on `cfg`, from one
+    committed ncu --set full capture (profiles/ncu_traffic.json), or None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(path) as f:
-            return json.load(f).get(cfg, {}).get("k_sweep_dram_bytes_per_launch")
+            d = json.load(f).get(cfg, {})
+        return d.get(f"{kernel}_dram_bytes_per_launch", d.get("k_sweep_dram_bytes_per_launch") if kernel == "k_sweep_da" else None)
     except Exception:
         return None
 
@@ -448,7 +451,7 @@ def main():
         achieved = 32.0 * blocks / kern_avg_s / 1e9
         peak = 128.0 * sms * sm_max * 1e6 / 1e9
         roofline = {"bound": "l1", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                    "traffic": ncu_traffic(cfg) if args.models == "rf" else None, "kernel": algo,
+                    "traffic": ncu_traffic(cfg, algo) if args.models == "rf" else None, "kernel": algo,
                     "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "algorithmic_bytes_per_launch": 32.0 * blocks,
                     "work": {"unit": "32-byte 2-level block fetches of the " +
@@ -468,7 +471,7 @@ def main():
         achieved = evals_step * dec / kern_avg_s / 1e9                  # G node-decisions / s
         peak = sms * sm_max * 1e6 * 32 / 2 / 1e9
         roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
-                    "frac": achieved / peak, "traffic": ncu_traffic(cfg) if args.models == "rf" else None,
+                    "frac": achieved / peak, "traffic": ncu_traffic(cfg, algo) if args.models == "rf" else None,
                     "kernel": algo, "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
                     "hbm": hbm, "per_kernel": per_kernel}

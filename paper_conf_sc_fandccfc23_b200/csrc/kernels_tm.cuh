@@ -59,9 +59,6 @@ struct TmArgs {
     int kb;                      // kernels per feature block (power of two, 32..256)
     int kb_log2;
     int fx32;                    // every forest's leaves are int32 fixed-point in its cut blocks
-    int ilv;                     // interleaved mode (small slabs): all slab features staged, CTA c
-                                 // takes chunks c, c + G, ... of (tree, 32-kernel group)
-    int ng;                      // 32-kernel groups in the slab (ilv)
     int nslot;                   // D slots = models with a forest member
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
@@ -86,133 +83,111 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
         sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
     }
-    const long long r0 = t.ilv ? 0 : (long long)blockIdx.x * t.n_tasks / gridDim.x;
-    const long long r1 = t.ilv ? 1 : (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
+    const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
+    const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
 
     const int lane = threadIdx.x & 31;
-    const unsigned xs_a = su32(xs);
     const unsigned xstride = 4u * (unsigned)KB;
     const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
     constexpr unsigned kEnt = 4u * NT;                                       // bytes between entries
     const int Fm1 = FR - 1;
 
     for (long long s0 = r0; s0 < r1;) {
-        const long long kbi = t.ilv ? 0 : s0 / per_kb;
-        const long long s1 = t.ilv ? r1 : min(r1, (kbi + 1) * per_kb);
+        const long long kbi = s0 / per_kb;
+        const long long s1 = min(r1, (kbi + 1) * per_kb);
         const int kbase = (int)(kbi * KB);                                   // slab-relative
         __syncthreads();                                                     // previous block done
         const float* gfeat = a.features + (t.slab0 + kbase) * F;
-        const int nvalid = min(KB, t.nks - kbase);                           // (ilv: KB = 32 * ng)
+        const int nvalid = min(KB, t.nks - kbase);
         for (int e = threadIdx.x; e < KB * F; e += NT) {
             const int kk = e / F, c = e - kk * F;
             xs[c * KB + kk] = kk < nvalid ? __ldg(gfeat + e) : 0.0f;
         }
         __syncthreads();
 
-        bool active = false, exhausted = false, lost = false;
-        const uint4* blocks = a.ms.blocks;
-        long long* drow = t.D;
-        double scale = 1.0;
-        unsigned xcol_a = xs_a;
-        int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
-        float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
-        long long vprev = 0;
-        // Static lane streams: task j belongs to lane j % 32 and warp (j / 32) % NW, so a lane's
-        // kernel-in-block kk = j % KB is always = lane (mod 32) and its feature reads hit its own
-        // bank (no conflicts, no shared counter); consecutive 32-task groups (one tree, 32
-        // kernels) go to consecutive warps.
-        // Interleaved mode: chunk ch = (tree ch / ng, kernel group ch % ng) of 32 tasks; CTA c's
-        // warp w takes chunks c + G * (w + NW * m), lane L its kernel 32 * group + L.
-        const int seg0 = (int)(s0 - kbi * per_kb), seg1 = t.ilv ? TT * t.ng : (int)(s1 - kbi * per_kb);
-        int q;                                                                // this lane's next offset
-        int qstep = NT;                                                       // 32 * NW
+        // Static lane streams: task j (tree j / KB, kernel-in-block j % KB) of the segment goes to
+        // lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same kernel kk
+        // (= lane mod 32: conflict-free feature reads) and its trees advance by NT / KB.
+        const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);
+        int q;
         {
             const int nw = NT / 32, w = threadIdx.x >> 5;
-            if (t.ilv) {
-                q = blockIdx.x + gridDim.x * w;                               // chunk index
-                qstep = gridDim.x * nw;
-            } else {
-                const int g0 = seg0 >> 5;
-                int g = g0 + ((w - g0 % nw) + nw) % nw;
-                q = 32 * g + lane;
-                if (q < seg0) q += 32 * nw;
-            }
+            const int g0 = seg0 >> 5;
+            const int g = g0 + ((w - g0 % nw) + nw) % nw;
+            q = 32 * g + lane;
+            if (q < seg0) q += NT;
         }
-        while (true) {
-            if (!active && !exhausted) {
-                // refill: this lane's next task of the segment
-                while (q < seg1) {
-                    int tti, kk;
-                    if (t.ilv) {
-                        tti = q / t.ng;
-                        kk = 32 * (q - tti * t.ng) + lane;
-                    } else {
-                        tti = q >> t.kb_log2;
-                        kk = q & (KB - 1);
-                    }
-                    q += qstep;
-                    if (kk >= nvalid) continue;
-                    const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
-                    const DevModel& m = da_model(a, mi);
-                    blocks = m.blocks;
-                    scale = m.fx_scale;
-                    root = sroot[tti];
-                    drow = t.D + ((kbase + kk) * t.nslot + t.slot_of[mi]) * n_f;
-                    xcol_a = xs_a + 4u * (unsigned)kk;
-                    bk = root;
-                    lo = 0;
-                    f_lo = 0.5f;
-                    tmin = CUDART_INF_F;
-                    sn = 0;
-                    lost = false;
-                    vprev = 0;
-                    active = true;
-                    break;
-                }
-                if (!active) exhausted = true;
-            }
-            if (__all_sync(0xffffffffu, exhausted)) break;
+        const int kk = q & (KB - 1);
+        const unsigned xcol_a = su32(xs) + 4u * (unsigned)kk;
+        long long* const dbase = t.D + (size_t)(kbase + kk) * t.nslot * n_f;
+        const uint4* blocks = a.ms.blocks;
+        long long* drow = dbase;
+        double scale = 1.0;
+        int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
+        bool lost = false;
+        float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
+        long long vprev = 0;
+        bool active = kk < nvalid && q < seg1;
+        // start the task at offset q (tree q / KB of this lane's kernel)
+        auto start = [&](int qq) {
+            const int tti = qq >> t.kb_log2;
+            const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
+            const DevModel& m = da_model(a, mi);
+            blocks = m.blocks;
+            scale = m.fx_scale;
+            root = sroot[tti];
+            drow = dbase + t.slot_of[mi] * n_f;
+            bk = root;
+            lo = 0;
+            f_lo = 0.5f;
+            tmin = CUDART_INF_F;
+            sn = 0;
+            lost = false;
+            vprev = 0;
+        };
+        if (active) start(q);
+        while (__any_sync(0xffffffffu, active)) {
             if (active) {
-                // one 2-level block step (internal.h layout), branch-free; cb = smallest cut of
-                // this block's left-turn clock splits.  Static features are read at a clamped
-                // row whatever the code, then selected.
-                uint4 A, B;
-                const int cur = bk;
-                ldg_blk256(blocks + 2 * (size_t)cur, A, B);
-                const unsigned codes = A.w;
-                const int cn = (int)(codes & 0xffu);
-                const float xs_n = lds_f(xcol_a + xstride * (unsigned)min(cn, Fm1));
-                const float xn = cn == F ? f_lo : xs_n;
-                const bool l0 = xn <= __uint_as_float(A.x);
-                float cb = (cn == F && l0) ? __uint_as_float(A.x) : CUDART_INF_F;
-                const unsigned tcb = l0 ? A.y : A.z;
-                const int cc = (int)((codes >> (l0 ? 8 : 16)) & 0xffu);
-                const float xs_c = lds_f(xcol_a + xstride * (unsigned)min(cc, Fm1));
-                const float xc = cc == F ? f_lo : xs_c;
-                const bool l1 = xc <= __uint_as_float(tcb);
-                if (cc == F && l1) cb = fminf(cb, __uint_as_float(tcb));
-                const unsigned g = l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
-                const int slot = (l0 ? 0 : 2) + (l1 ? 0 : 1);
-                const bool leaf_n = cn > F, leaf_c = cc > F;
-                const bool at_leaf = leaf_n || leaf_c || ((codes >> (24 + slot)) & 1u);
-                const unsigned leafbits = leaf_n ? A.x : leaf_c ? tcb : g;   // one-leaf / child / grandchild
-                bk = (int)g;
-                if (cb < tmin) {                                             // new record: push
-                    sts_u(sb_a + kEnt * (unsigned)wp, (unsigned)cur);
-                    sts_f(sc_a + kEnt * (unsigned)wp, cb);
-                    wp = (wp + 1) & (kTmS - 1);
-                    lost = lost || sn == kTmS;
-                    sn = min(sn + 1, kTmS);
-                    tmin = cb;
-                }
-                if (at_leaf) {
-                    // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
-                    const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
-                    const long long v = t.fx32 ? (long long)(int)leafbits     // int32 fixed point
-                                               : __double2ll_rn(__dmul_rn((double)__uint_as_float(leafbits), scale));
-                    atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
-                    vprev = v;
-                    active = hi < n_f;
+            // one 2-level block step (internal.h layout), branch-free; cb = smallest cut of this
+            // block's left-turn clock splits.  Static features are read at a clamped row whatever
+            // the code, then selected.
+            uint4 A, B;
+            const int cur = bk;
+            ldg_blk256(blocks + 2 * (size_t)cur, A, B);
+            const unsigned codes = A.w;
+            const int cn = (int)(codes & 0xffu);
+            const float xs_n = lds_f(xcol_a + xstride * (unsigned)min(cn, Fm1));
+            const float xn = cn == F ? f_lo : xs_n;
+            const bool l0 = xn <= __uint_as_float(A.x);
+            float cb = (cn == F && l0) ? __uint_as_float(A.x) : CUDART_INF_F;
+            const unsigned tcb = l0 ? A.y : A.z;
+            const int cc = (int)((codes >> (l0 ? 8 : 16)) & 0xffu);
+            const float xs_c = lds_f(xcol_a + xstride * (unsigned)min(cc, Fm1));
+            const float xc = cc == F ? f_lo : xs_c;
+            const bool l1 = xc <= __uint_as_float(tcb);
+            if (cc == F && l1) cb = fminf(cb, __uint_as_float(tcb));
+            const unsigned g = l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
+            const int slot = (l0 ? 0 : 2) + (l1 ? 0 : 1);
+            const bool leaf_n = cn > F, leaf_c = cc > F;
+            const bool at_leaf = leaf_n || leaf_c || ((codes >> (24 + slot)) & 1u);
+            const unsigned leafbits = leaf_n ? A.x : leaf_c ? tcb : g;       // one-leaf / child / grandchild
+            bk = (int)g;
+            if (cb < tmin) {                                                 // new record: push
+                sts_u(sb_a + kEnt * (unsigned)wp, (unsigned)cur);
+                sts_f(sc_a + kEnt * (unsigned)wp, cb);
+                wp = (wp + 1) & (kTmS - 1);
+                lost = lost || sn == kTmS;
+                sn = min(sn + 1, kTmS);
+                tmin = cb;
+            }
+            if (at_leaf) {
+                // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
+                const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
+                const long long v = t.fx32 ? (long long)(int)leafbits         // int32 fixed point
+                                           : __double2ll_rn(__dmul_rn((double)__uint_as_float(leafbits), scale));
+                atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
+                vprev = v;
+                if (hi < n_f) {
                     // resume at the top record's block (popped); a stack emptied after dropping
                     // shallower records restarts at the root
                     wp = (wp + kTmS - 1) & (kTmS - 1);
@@ -225,7 +200,12 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                     }
                     lo = hi;
                     f_lo = (float)hi + 0.5f;
+                } else {
+                    q += NT;                                                 // next tree, same kernel
+                    active = q < seg1;
+                    if (active) start(q);
                 }
+            }
             }
         }
         s0 = s1;

@@ -512,22 +512,11 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     t.kb = kb;
     t.kb_log2 = 0;
     while ((1 << t.kb_log2) < kb) ++t.kb_log2;
-    // interleaved mode (SYNERGY_TM_ILV=1, needs the whole slab's features in shared memory): every
-    // CTA mixes chunks of all trees.  Off by default: measured slower than contiguous ranges on
-    // c1/c2 (round 1), the L1 then holds many more trees.
-    const long long ngall = (n_k + 31) / 32;
-    t.ilv = env_int("SYNERGY_TM_ILV", 0) ? 1 : 0;
-    if (t.ilv && (size_t)std::max(F, 1) * ngall * 32 * 4 > 160 * 1024) t.ilv = 0;
-    if (t.ilv) {
-        t.kb = (int)(ngall * 32);
-        t.kb_log2 = 0;
-    }
     const size_t row = (size_t)t.nslot * n_f * sizeof(long long);
     // kernels per slab: a multiple of the feature block, D of one slab <= kTmSlabBytes (L2-resident)
     long long nks = std::max<long long>(kb, (long long)(kTmSlabBytes / row) / kb * kb);
     const int slab_env = env_int("SYNERGY_TM_SLAB", 0);
     if (slab_env > 0) nks = std::max<long long>(kb, slab_env / kb * kb);
-    if (t.ilv && slab_env <= 0) nks = n_k;                 // one slab: all features staged
     nks = std::min<long long>(nks, n_k);
     TmBuf* buf = nullptr;
     syn_status s = tm_buffer(device, st, (size_t)nks * row, &buf);
@@ -570,7 +559,6 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         t.slab0 = s0;
         t.nks = (int)std::min<long long>(nks, n_k - s0);
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * kb;
-        t.ng = (t.nks + 31) / 32;
         const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
         {
             KernelTimer ktm("k_tm_walk", st);

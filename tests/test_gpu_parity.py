@@ -26,8 +26,6 @@ def _build():
 #   tm_kb32   k_tm_walk with 32-kernel feature blocks (several blocks per CTA range)
 #   tm_ctas3  k_tm_walk on 3 CTAs (long per-CTA ranges crossing kernel blocks, many tasks/lane)
 #   tm_slab   kernel slabs of 64 (several walk + finish launches reusing the zeroed D buffer)
-#   tm_static contiguous per-CTA task ranges (the large-batch mode) on every size
-#   tm_ilv_slab interleaved chunks (the small-batch mode) with slabs of 96 kernels
 #   da        order-free difference-array kernel (k_sweep_da), shared-memory int64 sums
 #   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
 #   da_nt256  k_sweep_da with 256 threads per CTA
@@ -46,8 +44,7 @@ def _build():
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
 DA = {"SYNERGY_ALGO": "da"}
 VARIANTS = {"default": {}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
-            "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32", "SYNERGY_TM_ILV": "0"},
-            "tm_static": {"SYNERGY_TM_ILV": "0"}, "tm_ilv_slab": {"SYNERGY_TM_ILV": "1", "SYNERGY_TM_SLAB": "96"},
+            "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
             "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
             "da_kpc5": {**DA, "SYNERGY_KPC": "5"}, "da_nsub3": {**DA, "SYNERGY_NSUB": "3"},
             "da_nsub64": {**DA, "SYNERGY_NSUB": "64", "SYNERGY_KPC": "2"},
@@ -59,7 +56,7 @@ VARIANTS = {"default": {}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYN
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_TM_ILV", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+KNOBS = ("SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
