@@ -58,7 +58,6 @@ struct TmArgs {
     int nks;                     // kernels in this slab
     int kb;                      // kernels per feature block (power of two, 32..256)
     int kb_log2;
-    int fx32;                    // every forest's leaves are int32 fixed-point in its cut blocks
     int nslot;                   // D slots = models with a forest member
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
@@ -123,6 +122,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const uint4* blocks = a.ms.blocks;
         long long* drow = dbase;
         double scale = 1.0;
+        bool fxm = false;                                                    // this model's leaves are int32
         int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
         bool lost = false;
         float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
@@ -135,6 +135,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             const DevModel& m = da_model(a, mi);
             blocks = m.blocks;
             scale = m.fx_scale;
+            fxm = m.fx32 != 0;                                               // as k_cut_blocks converted them
             root = sroot[tti];
             drow = dbase + t.slot_of[mi] * n_f;
             bk = root;
@@ -183,7 +184,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             if (at_leaf) {
                 // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
                 const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
-                const long long v = t.fx32 ? (long long)(int)leafbits         // int32 fixed point
+                const long long v = fxm ? (long long)(int)leafbits            // int32 fixed point
                                            : __double2ll_rn(__dmul_rn((double)__uint_as_float(leafbits), scale));
                 atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
                 vprev = v;

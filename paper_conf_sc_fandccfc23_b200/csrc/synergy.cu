@@ -500,9 +500,6 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         tt += d.n_trees;
     }
     t.nm = nm;
-    t.fx32 = 1;
-    for (int m = 0; m < nm; ++m)
-        if (t.slot_of[m] >= 0 && !dms[m]->fx32) t.fx32 = 0;
     // kernels per feature block: a power of two in [32, 256], F * kb floats of shared memory
     int kb = 256;
     while (kb > 32 && ((size_t)F * kb * 4 > 32768 || kb / 2 >= n_k)) kb /= 2;

@@ -30,7 +30,7 @@ for s in $STAGES; do
       tail -5 $OUT/launches_c2.csv ;;
     full)
       for c in ${NCU_CFGS:-c2}; do
-        timeout 1200 ncu --set full --clock-control none --import-source on -k regex:k_sweep -s 3 -c 1 \
+        timeout 1200 ncu --set full --clock-control none --import-source on -k regex:${NCU_K:-k_tm_walk} -s 3 -c 1 \
           -o $OUT/prof_$c -f python bench.py --config $c --steps 2 --warmup 1 --no-cpu-baseline --no-e2e > $OUT/ncu_full_$c.log 2>&1
         tail -3 $OUT/ncu_full_$c.log
       done ;;

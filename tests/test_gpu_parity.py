@@ -137,9 +137,11 @@ def _stump_models(values_S, values_E, F=3):
     return w
 
 
-def test_exact_sum_where_sequential_fp64_rounds():
-    """Leaves spanning 2^24 .. 2^-30 ulps: the int64 path (k_sweep_da) is exact like the oracle,
-    while a sequential fp64 sum of these leaves rounds (Q8)."""
+@pytest.mark.parametrize("swap", [False, True])
+def test_exact_sum_where_sequential_fp64_rounds(swap):
+    """Leaves spanning 2^24 .. 2^-30 ulps: the int64 path is exact like the oracle, while a
+    sequential fp64 sum of these leaves rounds (Q8).  One model needs int64 leaves, the
+    other has int32 fixed-point leaves (both orders): each model's leaves are decoded its own way."""
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
     big = float(np.float32(2.0 ** 24 + 2.0))
     vals = [big, 0.008606708608567715, -big, 0.008446695283055305, big, 0.008703862316906452]
@@ -149,7 +151,7 @@ def test_exact_sum_where_sequential_fp64_rounds():
     for v in vals:
         seq += v
     assert seq != math.fsum(vals)                             # the case really needs exactness
-    w = _stump_models(vals, [1.0, 2.0])
+    w = _stump_models([1.0, 2.0], vals) if swap else _stump_models(vals, [1.0, 2.0])
     S, E = gpu_predict(w, default_idx=-1)
     rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
     assert syn.last_launch()["variant"] // 1000 in (3, 4)     # an exact int64 kernel ran
