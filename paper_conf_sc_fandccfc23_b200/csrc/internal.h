@@ -37,6 +37,7 @@ struct DevModel {
     const uint4* blocks;
     const int* broot;        // [n_trees] root block of each tree
     int bdepth;              // max(1, ceil(depth / 2)) over all trees
+    int nblk;                // blocks of all trees (tree t owns [broot[t], broot[t+1] or nblk))
     // exact fixed-point leaf sums (k_sweep_da): every leaf v is an integer multiple of 2^-s and
     // n_trees * max|v| * 2^s < 2^62, so v * fx_scale is an exact int64 and sums are exact
     int fx_ok;

@@ -21,9 +21,10 @@
 //    turn with a larger cut stays left).  So each lane keeps the prefix-minimum ("record") cuts
 //    of its path with their blocks, one entry per block, deepest on top: the next walk resumes at
 //    the top record's block (popped; the block is re-decided), and the new bound is the next
-//    record.  The stack keeps the kTmS deepest records; if it empties after shallower records
-//    were dropped, the walk restarts at the root.  On the bench forests this fetches 0.47x the
-//    blocks of root restarts.
+//    record.  The stack keeps the kTmS shallowest records (a depth-12 path has at most 6 blocks);
+//    deeper ones are not pushed, which stays exact: resuming at any ancestor block of the path
+//    re-walks the same path down to the split where clock hi turns right.  On the bench forests
+//    this fetches 0.47x the blocks of root restarts.
 //
 //  * Clock cuts instead of clock values.  For a given clock table every clock-split threshold
 //    thr is replaced (k_cut_blocks, once per (model, clock table)) by its cut index
@@ -34,7 +35,9 @@
 //
 //  * Step-level lockstep.  Every loop iteration is one 2-level block step for every busy lane; a
 //    lane that reaches a leaf closes its run and resumes in the same iteration, so walks of
-//    different lengths do not idle lanes.
+//    different lengths do not idle lanes.  Each lane keeps its kernel's features in its own
+//    shared-memory column with the walked clock as row F, so every split reads x[code] with no
+//    clock/feature select, and clock splits and leaves are flagged in the block (k_cut_blocks).
 //
 //  * Accumulation in L2.  Run j of a (kernel, model, tree) adds v_j - v_{j-1} to
 //    D[kernel][slot][lo_j] with one 64-bit global reduction (exact, order-free; run 0 adds v_0).
@@ -47,8 +50,17 @@
 
 namespace syn {
 
-constexpr int kTmS = 4;          // resume-stack entries per lane (shallowest kept)
+constexpr int kTmS = 6;          // record-stack entries per lane (a depth-12 path has <= 6 blocks)
 constexpr int kTmNT = 512;       // k_tm_walk threads per CTA (2 CTAs per SM)
+
+// Clock-cut block words (k_cut_blocks output; the layout of internal.h with two additions):
+//   word 3 bits 28/29/30: node / child 0 / child 1 splits on the clock (code == F)
+//   leaves folded into grandchild slots: a child that is a leaf (code F + 1) has both its
+//   grandchild slots set to its value with their leafmask bits, and a one-leaf tree has all four
+//   (children then read feature row F + 1 of any value: both outcomes reach the same leaf).
+// So a step reaches a leaf exactly when the leafmask bit of the slot it takes is set, and the
+// leaf value is that slot's word.
+constexpr unsigned kClkN = 1u << 28, kClkC0 = 1u << 29, kClkC1 = 1u << 30;
 
 struct TmArgs {
     SweepArgs s;                 // models, clocks, targets, outputs of the whole call
@@ -63,16 +75,41 @@ struct TmArgs {
     int nm;                      // models in the call (2 or 4)
 };
 
+// One 2-level block step on clock-cut words (A = {thr(n), thr(c0), thr(c1), codes}, grandchild
+// words B): the three candidate inputs are read from the lane's column xcol ([F + 2] rows of
+// stride NT: the kernel's static features, the walked clock in row F, row F + 1 for folded
+// leaves), then decided.  Returns the grandchild word taken; *cb = smallest cut of the block's
+// left-turn clock splits (+inf if none), *leaf = the word is a leaf value.
+template <int NT>
+__device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, const float* xcol, float& cb, bool& leaf) {
+    const unsigned codes = A.w;
+    const float xn = xcol[(size_t)(codes & 0xffu) * NT];
+    const float x0 = xcol[(size_t)((codes >> 8) & 0xffu) * NT];
+    const float x1 = xcol[(size_t)((codes >> 16) & 0xffu) * NT];
+    const bool l0 = xn <= __uint_as_float(A.x);
+    const unsigned tcb = l0 ? A.y : A.z;
+    const bool l1 = (l0 ? x0 : x1) <= __uint_as_float(tcb);
+    const float cbn = (l0 && (codes & kClkN)) ? __uint_as_float(A.x) : CUDART_INF_F;
+    const float cbc = (l1 && (codes & (l0 ? kClkC0 : kClkC1))) ? __uint_as_float(tcb) : CUDART_INF_F;
+    cb = fminf(cbn, cbc);
+    const int slot = (l0 ? 0 : 2) + (l1 ? 0 : 1);
+    leaf = (codes >> (24 + slot)) & 1u;
+    return l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
+}
+
 template <int NT>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
     extern __shared__ __align__(16) unsigned char smem[];
     const int n_f = a.n_f, F = a.F, KB = t.kb;
-    const int FR = max(F, 1);                                                // feature rows staged
     int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
-    float* xs = stk_c + kTmS * NT;                                           // [FR][KB] features
-    int* sroot = reinterpret_cast<int*>(xs + (size_t)FR * KB);              // [TT] root block per tree
+    float* xs = stk_c + kTmS * NT;                                           // [F + 2][NT] lane columns
+    int* sroot = reinterpret_cast<int*>(xs + (size_t)(F + 2) * NT);         // [TT] root block per tree
+    int* const sb = stk_b + threadIdx.x;
+    float* const sc = stk_c + threadIdx.x;
+    float* const xcol = xs + threadIdx.x;
+    float* const xclk = xcol + (size_t)F * NT;
 
     const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
               T3 = t.nm > 2 ? da_trees(a, 3) : 0;
@@ -82,31 +119,20 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
         sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
     }
+    __syncthreads();
     const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
     const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
-
     const int lane = threadIdx.x & 31;
-    const unsigned xstride = 4u * (unsigned)KB;
-    const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
-    constexpr unsigned kEnt = 4u * NT;                                       // bytes between entries
-    const int Fm1 = FR - 1;
 
     for (long long s0 = r0; s0 < r1;) {
         const long long kbi = s0 / per_kb;
         const long long s1 = min(r1, (kbi + 1) * per_kb);
         const int kbase = (int)(kbi * KB);                                   // slab-relative
-        __syncthreads();                                                     // previous block done
-        const float* gfeat = a.features + (t.slab0 + kbase) * F;
         const int nvalid = min(KB, t.nks - kbase);
-        for (int e = threadIdx.x; e < KB * F; e += NT) {
-            const int kk = e / F, c = e - kk * F;
-            xs[c * KB + kk] = kk < nvalid ? __ldg(gfeat + e) : 0.0f;
-        }
-        __syncthreads();
 
         // Static lane streams: task j (tree j / KB, kernel-in-block j % KB) of the segment goes to
-        // lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same kernel kk
-        // (= lane mod 32: conflict-free feature reads) and its trees advance by NT / KB.
+        // lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same kernel kk and its
+        // trees advance by NT / KB: the lane's feature column is loaded once per segment.
         const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);
         int q;
         {
@@ -117,17 +143,19 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             if (q < seg0) q += NT;
         }
         const int kk = q & (KB - 1);
-        const unsigned xcol_a = su32(xs) + 4u * (unsigned)kk;
         long long* const dbase = t.D + (size_t)(kbase + kk) * t.nslot * n_f;
         const uint4* blocks = a.ms.blocks;
         long long* drow = dbase;
         double scale = 1.0;
         bool fxm = false;                                                    // this model's leaves are int32
-        int root = 0, bk = 0, lo = 0, sn = 0, wp = 0;
-        bool lost = false;
-        float f_lo = 0.5f, tmin = CUDART_INF_F;                             // clock lo enters as lo + 0.5
+        int bk = 0, lo = 0, sn = 0;
+        float tmin = CUDART_INF_F;
         long long vprev = 0;
         bool active = kk < nvalid && q < seg1;
+        if (active) {
+            const float* g = a.features + (t.slab0 + kbase + kk) * F;
+            for (int c = 0; c < F; ++c) xcol[(size_t)c * NT] = __ldg(g + c);
+        }
         // start the task at offset q (tree q / KB of this lane's kernel)
         auto start = [&](int qq) {
             const int tti = qq >> t.kb_log2;
@@ -136,86 +164,61 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             blocks = m.blocks;
             scale = m.fx_scale;
             fxm = m.fx32 != 0;                                               // as k_cut_blocks converted them
-            root = sroot[tti];
+            bk = sroot[tti];
             drow = dbase + t.slot_of[mi] * n_f;
-            bk = root;
             lo = 0;
-            f_lo = 0.5f;
+            *xclk = 0.5f;                                                    // clock lo enters as lo + 0.5
             tmin = CUDART_INF_F;
             sn = 0;
-            lost = false;
             vprev = 0;
         };
         if (active) start(q);
         while (__any_sync(0xffffffffu, active)) {
-            if (active) {
-            // one 2-level block step (internal.h layout), branch-free; cb = smallest cut of this
-            // block's left-turn clock splits.  Static features are read at a clamped row whatever
-            // the code, then selected.
+            if (!active) continue;
             uint4 A, B;
             const int cur = bk;
             ldg_blk256(blocks + 2 * (size_t)cur, A, B);
-            const unsigned codes = A.w;
-            const int cn = (int)(codes & 0xffu);
-            const float xs_n = lds_f(xcol_a + xstride * (unsigned)min(cn, Fm1));
-            const float xn = cn == F ? f_lo : xs_n;
-            const bool l0 = xn <= __uint_as_float(A.x);
-            float cb = (cn == F && l0) ? __uint_as_float(A.x) : CUDART_INF_F;
-            const unsigned tcb = l0 ? A.y : A.z;
-            const int cc = (int)((codes >> (l0 ? 8 : 16)) & 0xffu);
-            const float xs_c = lds_f(xcol_a + xstride * (unsigned)min(cc, Fm1));
-            const float xc = cc == F ? f_lo : xs_c;
-            const bool l1 = xc <= __uint_as_float(tcb);
-            if (cc == F && l1) cb = fminf(cb, __uint_as_float(tcb));
-            const unsigned g = l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
-            const int slot = (l0 ? 0 : 2) + (l1 ? 0 : 1);
-            const bool leaf_n = cn > F, leaf_c = cc > F;
-            const bool at_leaf = leaf_n || leaf_c || ((codes >> (24 + slot)) & 1u);
-            const unsigned leafbits = leaf_n ? A.x : leaf_c ? tcb : g;       // one-leaf / child / grandchild
+            float cb;
+            bool at_leaf;
+            const unsigned g = tm_step<NT>(A, B, xcol, cb, at_leaf);
             bk = (int)g;
-            if (cb < tmin) {                                                 // new record: push
-                sts_u(sb_a + kEnt * (unsigned)wp, (unsigned)cur);
-                sts_f(sc_a + kEnt * (unsigned)wp, cb);
-                wp = (wp + 1) & (kTmS - 1);
-                lost = lost || sn == kTmS;
-                sn = min(sn + 1, kTmS);
+            if (cb < tmin) {                                                 // new record
+                if (sn < kTmS) {                                             // deeper ones are not kept:
+                    sb[sn * NT] = cur;                                       // resuming at an ancestor on
+                    sc[sn * NT] = cb;                                        // the path is still exact
+                    ++sn;
+                }
                 tmin = cb;
             }
             if (at_leaf) {
                 // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
                 const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
-                const long long v = fxm ? (long long)(int)leafbits            // int32 fixed point
-                                           : __double2ll_rn(__dmul_rn((double)__uint_as_float(leafbits), scale));
+                const long long v = fxm ? (long long)(int)g
+                                        : __double2ll_rn(__dmul_rn((double)__uint_as_float(g), scale));
                 atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
                 vprev = v;
                 if (hi < n_f) {
-                    // resume at the top record's block (popped); a stack emptied after dropping
-                    // shallower records restarts at the root
-                    wp = (wp + kTmS - 1) & (kTmS - 1);
-                    bk = (int)lds_u(sb_a + kEnt * (unsigned)wp);
+                    // resume at the deepest kept record's block (popped); the next one is the bound
                     --sn;
-                    tmin = sn > 0 ? lds_f(sc_a + kEnt * (unsigned)((wp + kTmS - 1) & (kTmS - 1))) : CUDART_INF_F;
-                    if (sn == 0 && lost) {
-                        bk = root;
-                        lost = false;
-                    }
+                    bk = sb[sn * NT];
+                    tmin = sn > 0 ? sc[(sn - 1) * NT] : CUDART_INF_F;
                     lo = hi;
-                    f_lo = (float)hi + 0.5f;
+                    *xclk = (float)hi + 0.5f;
                 } else {
                     q += NT;                                                 // next tree, same kernel
                     active = q < seg1;
                     if (active) start(q);
                 }
             }
-            }
         }
         s0 = s1;
     }
 }
 
-// Clock-specialised copy of a model's 2-level blocks (see the header): every clock-split
-// threshold (code == F) becomes its cut index #{i : f_i <= thr} as an fp32 integer.  One thread
-// per block; child-leaf values (code F + 1) and grandchild slots are copied unchanged.
+// Clock-specialised copy of a model's 2-level blocks (see the header and kClkN above): every
+// clock-split threshold (code == F) becomes its cut index #{i : f_i <= thr} as an fp32 integer,
+// leaves become int32 fixed point when the model allows, clock splits are flagged and leaves are
+// folded into grandchild slots.  One thread per block.
 __global__ void __launch_bounds__(256) k_cut_blocks(const uint4* __restrict__ in, long long n_blocks, int F,
                                                     const float* __restrict__ freqs, int n_f,
                                                     double fx_scale, uint4* __restrict__ out) {
@@ -225,15 +228,16 @@ __global__ void __launch_bounds__(256) k_cut_blocks(const uint4* __restrict__ in
     const uint4 B = in[2 * b + 1];
     unsigned w[3] = {A.x, A.y, A.z};
     unsigned g[4] = {B.x, B.y, B.z, B.w};
+    int code[3];
 #pragma unroll
     for (int q = 0; q < 3; ++q) {
-        const int code = (int)((A.w >> (8 * q)) & 0xffu);
-        if (code > F && fx_scale != 0.0) {
+        code[q] = (int)((A.w >> (8 * q)) & 0xffu);
+        if (code[q] > F && fx_scale != 0.0) {
             // leaf value (one-leaf tree at q = 0, child leaf at q = 1, 2) -> int32 v * 2^s, exact
             w[q] = (unsigned)__double2int_rn(__dmul_rn((double)__uint_as_float(w[q]), fx_scale));
             continue;
         }
-        if (code != F) continue;
+        if (code[q] != F) continue;
         const float thr = __uint_as_float(w[q]);
         int l = 0, h = n_f;                                  // #{i : f_i <= thr}
         while (l < h) {
@@ -242,14 +246,25 @@ __global__ void __launch_bounds__(256) k_cut_blocks(const uint4* __restrict__ in
         }
         w[q] = __float_as_uint((float)l);
     }
+    unsigned lm = (A.w >> 24) & 0xfu;
     if (fx_scale != 0.0) {
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-            if ((A.w >> (24 + q)) & 1u) g[q] = (unsigned)__double2int_rn(__dmul_rn((double)__uint_as_float(g[q]), fx_scale));
+            if ((lm >> q) & 1u) g[q] = (unsigned)__double2int_rn(__dmul_rn((double)__uint_as_float(g[q]), fx_scale));
+    }
+    if (code[0] > F) {                                       // one-leaf tree
+        code[1] = code[2] = F + 1;
+        g[0] = g[1] = g[2] = g[3] = w[0];
+        lm = 0xfu;
+    } else {
+        if (code[1] > F) { g[0] = g[1] = w[1]; lm |= 3u; }
+        if (code[2] > F) { g[2] = g[3] = w[2]; lm |= 12u; }
     }
     A.x = w[0];
     A.y = w[1];
     A.z = w[2];
+    A.w = (unsigned)code[0] | ((unsigned)code[1] << 8) | ((unsigned)code[2] << 16) | (lm << 24) |
+          (code[0] == F ? kClkN : 0u) | (code[1] == F ? kClkC0 : 0u) | (code[2] == F ? kClkC1 : 0u);
     out[2 * b] = A;
     out[2 * b + 1] = make_uint4(g[0], g[1], g[2], g[3]);
 }

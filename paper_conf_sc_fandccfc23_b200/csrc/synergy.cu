@@ -22,6 +22,7 @@
 #include "kernels_da.cuh"
 #include "kernels_svr.cuh"
 #include "kernels_tm.cuh"
+#include "kernels_tr.cuh"
 #include "synergy.h"
 
 using namespace syn;
@@ -37,6 +38,8 @@ struct syn_model {
     DevModel dm;
     long long n_blocks;                                   // 2-level blocks (2 x uint4 each)
     std::vector<std::pair<long long, uint4*>> cut_blocks;  // per clock table (uid): k_cut_blocks copy
+    std::vector<std::pair<long long, uint4*>> tr_blocks;   // per clock table (uid): k_tr_layout copy
+    long long max_tree_blocks;                            // blocks of the largest tree
 };
 
 struct syn_clocks {
@@ -387,6 +390,7 @@ cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaS
 struct TmBuf {
     int dev;
     cudaStream_t st;
+    int kind;                        // 0: D (kept all-zero between calls), 1: k_tr_walk features
     long long* p;
     size_t bytes;
     bool dirty;
@@ -394,13 +398,13 @@ struct TmBuf {
 std::mutex g_tm_mu;
 std::list<TmBuf> g_tm_bufs;          // list: entries never move
 
-syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out) {
+syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out, int kind = 0) {
     std::lock_guard<std::mutex> lock(g_tm_mu);
     TmBuf* b = nullptr;
     for (TmBuf& x : g_tm_bufs)
-        if (x.dev == dev && x.st == st) b = &x;
+        if (x.dev == dev && x.st == st && x.kind == kind) b = &x;
     if (!b) {
-        g_tm_bufs.push_back({dev, st, nullptr, 0, false});
+        g_tm_bufs.push_back({dev, st, kind, nullptr, 0, false});
         b = &g_tm_bufs.back();
     }
     cudaError_t e = cudaSuccess;
@@ -420,7 +424,7 @@ syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out) {
         b->bytes = bytes;
         b->dirty = true;
     }
-    if (b->dirty) {
+    if (b->dirty && kind == 0) {
         if ((e = cudaMemsetAsync(b->p, 0, b->bytes, st)) != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(D)");
         b->dirty = false;
     }
@@ -458,7 +462,34 @@ syn_status cut_blocks(syn_model* m, const syn_clocks* c, const uint4** out) {
     return ok();
 }
 
-constexpr size_t kTmSlabBytes = 48u << 20;   // D bytes per slab (stays L2-resident with the model)
+// Tree-resident copy (kernels_tr.cuh, k_tr_layout) of a model's clock-cut blocks, cached like them.
+syn_status tr_blocks(syn_model* m, const syn_clocks* c, const uint4* cut, const uint4** out) {
+    std::lock_guard<std::mutex> lock(g_cut_mu);
+    for (auto& cb : m->tr_blocks)
+        if (cb.first == c->uid) {
+            *out = cb.second;
+            return ok();
+        }
+    uint4* p = nullptr;
+    const long long nb = std::max<long long>(m->n_blocks, 1);
+    cudaError_t e = cudaMalloc(&p, (size_t)nb * 2 * sizeof(uint4));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return cuda_fail(e, "cudaMalloc(tree-resident blocks)");
+    }
+    if (m->n_trees > 0)
+        k_tr_layout<<<(unsigned)m->n_trees, 256>>>(cut, m->dm.broot, m->n_trees, m->n_blocks, p);
+    if ((e = cudaGetLastError()) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess) {
+        cudaFree(p);
+        return cuda_fail(e, "k_tr_layout");
+    }
+    m->tr_blocks.push_back({c->uid, p});
+    *out = p;
+    return ok();
+}
+
+constexpr size_t kTmSlabBytes = 48u << 20;
+constexpr size_t kTrTreeMax = 64u << 10;     // largest tree (bytes of 2-level blocks) k_tr_walk stages   // D bytes per slab (stays L2-resident with the model)
 
 // Tree-major path (k_tm_walk + k_tm_finish per kernel slab).  Needs every forest within the exact
 // int64 leaf range (fx_ok) and at least one tree; returns false (nothing enqueued) otherwise.
@@ -475,15 +506,30 @@ bool tm_eligible(const SweepArgs& a, int nm) {
 }
 
 syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clocks* clocks, cudaStream_t st,
-                  int* launches) {
+                  int* launches, int* variant) {
     const int device = clocks->device;
     DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
+    // k_tm_walk (trees read through L1) by default; SYNERGY_TM_MODE=tr selects the tree-resident
+    // k_tr_walk when every tree fits its shared tree buffer (measured slower on the bench
+    // forests: with two 44-KB tree buffers per SM the lanes wait for stragglers)
+    const char* mode_env = getenv("SYNERGY_TM_MODE");
+    bool use_tr = mode_env && !strcmp(mode_env, "tr");
+    long long max_tb = 1;
+    for (int m = 0; m < nm; ++m)
+        if (models[m] && dms[m]->forest_weight != 0.0 && dms[m]->n_trees > 0)
+            max_tb = std::max(max_tb, models[m]->max_tree_blocks);
+    if ((size_t)max_tb * 32 > kTrTreeMax) use_tr = false;
+    for (int m = 0; m < nm; ++m)                  // k_tr_walk decodes int32 fixed-point leaves only
+        if (models[m] && dms[m]->forest_weight != 0.0 && dms[m]->n_trees > 0 && !dms[m]->fx32) use_tr = false;
+    TrArgs r;
+    memset(&r, 0, sizeof r);
     for (int m = 0; m < nm; ++m) {
         if (!models[m] || dms[m]->forest_weight == 0.0 || dms[m]->n_trees == 0) continue;
         const uint4* cb = nullptr;
         syn_status cs = cut_blocks(models[m], clocks, &cb);
         if (cs != SYN_OK) return cs;
         dms[m]->blocks = cb;
+        if (use_tr && (cs = tr_blocks(models[m], clocks, cb, &r.trb[m])) != SYN_OK) return cs;
     }
     TmArgs t;
     memset(&t, 0, sizeof t);
@@ -515,10 +561,22 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     const int slab_env = env_int("SYNERGY_TM_SLAB", 0);
     if (slab_env > 0) nks = std::max<long long>(kb, slab_env / kb * kb);
     nks = std::min<long long>(nks, n_k);
+    // k_tr_walk chunk size P (kernels per unit): 1024, halved down to 512 while that leaves fewer
+    // than 4 units per SM; the slab's transposed features ride in the same scratch as D
+    const int sms_tr = sm_count(device);
+    int P = 1024;
+    while (P > 512 && (long long)tt * ((std::min<long long>(nks, n_k) + P - 1) / P) < 4LL * sms_tr) P /= 2;
+    const int p_env = env_int("SYNERGY_TR_P", P);
+    if (p_env >= 32 && p_env <= 2048 && p_env % 32 == 0) P = p_env;
     TmBuf* buf = nullptr;
     syn_status s = tm_buffer(device, st, (size_t)nks * row, &buf);
     if (s != SYN_OK) return s;
     t.D = buf->p;
+    if (use_tr && F > 0) {
+        TmBuf* fb = nullptr;
+        if ((s = tm_buffer(device, st, (size_t)((nks + P - 1) / P) * F * P * 4, &fb, 1)) != SYN_OK) return s;
+        r.featT = reinterpret_cast<const float*>(fb->p);
+    }
     // finish tile: KT kernels per CTA, fp64 + fp32 per (model, kernel, clock) in shared memory
     // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
     int kt = std::max(1, std::min(8, (int)((150 * 1024) / ((size_t)nm * n_f * 12 + (size_t)t.nslot * n_f * 8))));
@@ -528,7 +586,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     a.xs = (F + 2) | 1;
     const size_t fsmem = (size_t)nm * kt * n_f * 12 + (size_t)n_f * 4 + (size_t)kt * a.xs * 4 + 32 +
                          (size_t)kt * t.nslot * n_f * 8;
-    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)std::max(F, 1) * t.kb * 4 + 16 + (size_t)tt * 4;
+    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 4;
     static size_t fset = 48 * 1024, wset = 48 * 1024;
     cudaError_t e = cudaSuccess;
     if (fsmem > fset) {
@@ -550,21 +608,57 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         carve_set = carve;
     }
     const int ctas = std::max(1, env_int("SYNERGY_TM_CTAS", 2 * sm_count(device)));
+    // k_tr_walk: kTrNB tree buffers + the chunk's [F][P] features + record stacks
+    r.tree_smem = (int)(((size_t)max_tb * 32 + 127) / 128 * 128);
+    r.P = P;
+    const size_t rsmem = (size_t)kTrNB * r.tree_smem + (size_t)F * P * 4 + (size_t)kTmS * kTrNT * 8;
+    if (use_tr) {
+        static size_t rset = 48 * 1024;
+        if (rsmem > rset) {
+            if ((e = cudaFuncSetAttribute(k_tr_walk<kTrNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rsmem)) != cudaSuccess)
+                return cuda_fail(e, "k_tr_walk attribute");
+            rset = rsmem;
+        }
+    }
     t.s = a;
     int n = 0;
     for (long long s0 = 0; s0 < n_k; s0 += nks) {
         t.slab0 = s0;
         t.nks = (int)std::min<long long>(nks, n_k - s0);
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * kb;
-        const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
-        {
-            KernelTimer ktm("k_tm_walk", st);
-            k_tm_walk<kTmNT><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-            e = cudaGetLastError();
-        }
-        if (e != cudaSuccess) {
-            buf->dirty = true;
-            return cuda_fail(e, "k_tm_walk launch");
+        if (use_tr) {
+            // unit = (tree, chunk of P kernels), one CTA per SM over contiguous unit ranges
+            r.nchunks = (t.nks + P - 1) / P;
+            r.tm = t;
+            {
+                const long long nf = (long long)r.nchunks * F * P;
+                KernelTimer ktf("k_tr_feat", st);
+                if (nf > 0) k_tr_feat<<<(unsigned)((nf + 255) / 256), 256, 0, st>>>(a.features, t.slab0, t.nks, F, P, r.nchunks, const_cast<float*>(r.featT));
+                e = cudaGetLastError();
+            }
+            const long long units = (long long)r.nchunks * tt;
+            const long long g = std::max<long long>(1, std::min<long long>(env_int("SYNERGY_TR_CTAS", sms_tr), units));
+            if (e == cudaSuccess) {
+                KernelTimer ktm("k_tr_walk", st);
+                k_tr_walk<kTrNT><<<(unsigned)g, kTrNT, rsmem, st>>>(r);
+                e = cudaGetLastError();
+            }
+            if (e != cudaSuccess) {
+                buf->dirty = true;
+                return cuda_fail(e, "k_tr_walk launch");
+            }
+            ++n;
+        } else {
+            const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
+            {
+                KernelTimer ktm("k_tm_walk", st);
+                k_tm_walk<kTmNT><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+                e = cudaGetLastError();
+            }
+            if (e != cudaSuccess) {
+                buf->dirty = true;
+                return cuda_fail(e, "k_tm_walk launch");
+            }
         }
         {
             KernelTimer ktm("k_tm_finish", st);
@@ -578,6 +672,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         n += 2;
     }
     *launches = n;
+    *variant = use_tr ? 4001 : 4000;
     return ok();
 }
 
@@ -855,9 +950,11 @@ syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_fe
     if (!algo_env && tm_eligible(a, 2)) {
         int nl = 0;
         syn_model* ms[2] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en)};
-        ss = run_tm(a, 2, ms, clocks, st, &nl);
+        int var = 4000;
+        ss = run_tm(a, 2, ms, clocks, st, &nl, &var);
         if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k), kTmNT, 4000};
+        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k),
+                  var == 4001 ? kTrNT : kTmNT, var};
         return ok();
     }
     static const char* knames[4] = {"k_sweep", "k_sweep_iv", "k_sweep_ws", "k_sweep_da"};
@@ -1113,6 +1210,11 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
     m->dm.bdepth = bdepth;
     m->n_blocks = (long long)(blocks.size() >> 1);
+    m->dm.nblk = (int)m->n_blocks;
+    m->max_tree_blocks = 0;
+    for (size_t t = 0; t < broot.size(); ++t)
+        m->max_tree_blocks = std::max<long long>(m->max_tree_blocks,
+                                                 (t + 1 < broot.size() ? broot[t + 1] : m->n_blocks) - broot[t]);
     m->dm.fx_ok = fx_ok;
     m->dm.fx32 = fx32;
     m->dm.fx_scale = std::ldexp(1.0, fx_s);
@@ -1139,6 +1241,7 @@ syn_status synergy_model_destroy(syn_model* m) {
         DeviceGuard g(m->device);
         cudaFree(m->alloc);
         for (auto& cb : m->cut_blocks) cudaFree(cb.second);
+        for (auto& cb : m->tr_blocks) cudaFree(cb.second);
     }
     delete m;
     return ok();
@@ -1304,9 +1407,11 @@ syn_status synergy_sweep4(const syn_model* const* models, const float* d_feature
         int nl = 0;
         syn_model* ms[4] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en), const_cast<syn_model*>(x2),
                             const_cast<syn_model*>(x3)};
-        ss = run_tm(a, 4, ms, clocks, st, &nl);
+        int var = 4000;
+        ss = run_tm(a, 4, ms, clocks, st, &nl, &var);
         if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k), kTmNT, 4000};
+        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k),
+                  var == 4001 ? kTrNT : kTmNT, var};
         return ok();
     }
     cudaError_t e;

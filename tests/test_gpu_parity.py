@@ -22,7 +22,11 @@ def _build():
 
 
 # Kernel variants the library can pick (read per call from the environment):
-#   default   tree-major resume walks (k_tm_walk + k_tm_finish), exact int64 leaf sums in L2
+#   default   tree-major resume walks through L1 (k_tm_walk + k_tm_finish), exact int64 sums in L2
+#   tr        tree-resident resume walks (k_tr_walk + k_tm_finish): trees and chunk features staged
+#             in shared memory by bulk copy, per-lane-index task pools (opt-in, SYNERGY_TM_MODE=tr)
+#   tr_p96    k_tr_walk with 96-kernel chunks (3 kernels per pool, most lanes draw nothing)
+#   tr_ctas3  k_tr_walk on 3 CTAs (many units and chunk switches per CTA: ring phases, restaging)
 #   tm_kb32   k_tm_walk with 32-kernel feature blocks (several blocks per CTA range)
 #   tm_ctas3  k_tm_walk on 3 CTAs (long per-CTA ranges crossing kernel blocks, many tasks/lane)
 #   tm_slab   kernel slabs of 64 (several walk + finish launches reusing the zeroed D buffer)
@@ -43,7 +47,9 @@ def _build():
 #   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
 #   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
 DA = {"SYNERGY_ALGO": "da"}
-VARIANTS = {"default": {}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
+TR = {"SYNERGY_TM_MODE": "tr"}
+VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
+            "tr_ctas3": {**TR, "SYNERGY_TR_CTAS": "3"}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
             "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
             "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
             "da_kpc5": {**DA, "SYNERGY_KPC": "5"}, "da_nsub3": {**DA, "SYNERGY_NSUB": "3"},
@@ -56,7 +62,7 @@ VARIANTS = {"default": {}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYN
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+KNOBS = ("SYNERGY_TM_MODE", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
@@ -121,6 +127,25 @@ def test_fuzz_bit_exact(case, variant):
         w.targets = tg
         ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
         got = gpu_sweep(w, want_pred=True)
+        assert_bits_equal(got["S"], ref["S"], "S")
+        assert_bits_equal(got["E"], ref["E"], "E")
+        assert_choices(got["choice"], ref["choice"], ref["gap"])
+
+
+def test_tree_resident_routing(monkeypatch):
+    """With SYNERGY_TM_MODE=tr, k_tr_walk (variant 4001) runs when every tree fits its 64 KB shared
+    tree buffer; a model with a larger tree routes to the L1-cached k_tm_walk (4000); both exact."""
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    for k in KNOBS:
+        monkeypatch.delenv(k, raising=False)
+    monkeypatch.setenv("SYNERGY_TM_MODE", "tr")
+    small = W.fuzz_workload(77, 40, 64, F=4, n_trees=3, max_depth=8, p_leaf=0.1)
+    big = W.fuzz_workload(78, 40, 64, F=4, n_trees=2, max_depth=16, p_freq=0.3, p_leaf=0.0)
+    assert max(np.diff(big.energy.tree_offset)) > 2 * 4 * 2048      # > 2048 2-level blocks
+    for w, want in ((small, 4001), (big, 4000)):
+        ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
+        got = gpu_sweep(w, want_pred=True)
+        assert syn.last_launch()["variant"] == want
         assert_bits_equal(got["S"], ref["S"], "S")
         assert_bits_equal(got["E"], ref["E"], "E")
         assert_choices(got["choice"], ref["choice"], ref["gap"])
