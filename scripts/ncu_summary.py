@@ -48,7 +48,7 @@ def raw(rep):
 
 def main():
     out, title, specs = sys.argv[1], sys.argv[2], sys.argv[3:]
-    cols = [(s.split("=", 1)[0], *raw(s.split("=", 1)[1])) for s in specs]
+    cols = [(s.rsplit("=", 1)[0], *raw(s.rsplit("=", 1)[1])) for s in specs]
     lines = [f"# {title}", "", "| metric | " + " | ".join(f"{c[0]} (`{c[1][:32]}`)" for c in cols) + " |",
              "|---|" + "---|" * len(cols)]
     for m in METRICS:
