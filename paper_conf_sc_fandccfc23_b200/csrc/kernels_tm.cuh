@@ -73,6 +73,7 @@ struct TmArgs {
     int nslot;                   // D slots = models with a forest member
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
+    int nsub;                    // clock sub-ranges per (kernel, tree) task (small batches)
 };
 
 // One 2-level block step on clock-cut words (A = {thr(n), thr(c0), thr(c1), codes}, grandchild
@@ -114,7 +115,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
               T3 = t.nm > 2 ? da_trees(a, 3) : 0;
     const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
-    const long long per_kb = (long long)TT * KB;
+    const int NS = t.nsub;
+    const long long per_kb = (long long)TT * NS * KB;
     for (int q = threadIdx.x; q < TT; q += NT) {
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
         sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
@@ -148,7 +150,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         long long* drow = dbase;
         double scale = 1.0;
         bool fxm = false;                                                    // this model's leaves are int32
-        int bk = 0, lo = 0, sn = 0;
+        int bk = 0, lo = 0, sn = 0, end = n_f;
         float tmin = CUDART_INF_F;
         long long vprev = 0;
         bool active = kk < nvalid && q < seg1;
@@ -156,9 +158,12 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             const float* g = a.features + (t.slab0 + kbase + kk) * F;
             for (int c = 0; c < F; ++c) xcol[(size_t)c * NT] = __ldg(g + c);
         }
-        // start the task at offset q (tree q / KB of this lane's kernel)
+        // start the task at offset q: tree (q / KB) / NS, clock sub-range (q / KB) % NS of this
+        // lane's kernel.  A sub-range [lo, end) walks from the root at clock lo and, at its end,
+        // takes its last value back out at D[end] so the difference arrays stay exact.
         auto start = [&](int qq) {
-            const int tti = qq >> t.kb_log2;
+            const int ts = qq >> t.kb_log2;
+            const int tti = NS == 1 ? ts : ts / NS, sub = ts - tti * NS;
             const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
             const DevModel& m = da_model(a, mi);
             blocks = m.blocks;
@@ -166,8 +171,9 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             fxm = m.fx32 != 0;                                               // as k_cut_blocks converted them
             bk = sroot[tti];
             drow = dbase + t.slot_of[mi] * n_f;
-            lo = 0;
-            *xclk = 0.5f;                                                    // clock lo enters as lo + 0.5
+            lo = NS == 1 ? 0 : sub * n_f / NS;                               // n_f <= 4096, NS <= 64
+            end = NS == 1 ? n_f : (sub + 1) * n_f / NS;
+            *xclk = (float)lo + 0.5f;                                        // clock lo enters as lo + 0.5
             tmin = CUDART_INF_F;
             sn = 0;
             vprev = 0;
@@ -197,7 +203,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                                         : __double2ll_rn(__dmul_rn((double)__uint_as_float(g), scale));
                 atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
                 vprev = v;
-                if (hi < n_f) {
+                if (hi < end) {
                     // resume at the deepest kept record's block (popped); the next one is the bound
                     --sn;
                     bk = sb[sn * NT];
@@ -205,7 +211,9 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                     lo = hi;
                     *xclk = (float)hi + 0.5f;
                 } else {
-                    q += NT;                                                 // next tree, same kernel
+                    if (end < n_f)                                           // sub-range end: D[end] -= v
+                        atomicAdd(reinterpret_cast<unsigned long long*>(drow + end), (unsigned long long)(-v));
+                    q += NT;                                                 // next task, same kernel
                     active = q < seg1;
                     if (active) start(q);
                 }
@@ -340,3 +348,4 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
 }
 
 }  // namespace syn
+

@@ -625,7 +625,15 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     for (long long s0 = 0; s0 < n_k; s0 += nks) {
         t.slab0 = s0;
         t.nks = (int)std::min<long long>(nks, n_k - s0);
-        t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * kb;
+        // tiny batches: split every (kernel, tree) task into clock sub-ranges while there are fewer
+        // tasks than resident lanes (at most 8 sub-ranges of at least 8 clocks; each sub-range
+        // adds a root descent, so batches with a task per lane keep whole tasks)
+        t.nsub = 1;
+        const long long lanes = (long long)ctas * kTmNT;
+        while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8) t.nsub *= 2;
+        const int ns_env = env_int("SYNERGY_TM_NSUB", t.nsub);
+        if (ns_env >= 1 && ns_env <= n_f && ns_env <= 64) t.nsub = ns_env;
+        t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * t.nsub * kb;
         if (use_tr) {
             // unit = (tree, chunk of P kernels), one CTA per SM over contiguous unit ranges
             r.nchunks = (t.nks + P - 1) / P;

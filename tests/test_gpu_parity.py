@@ -29,6 +29,8 @@ def _build():
 #   tr_ctas3  k_tr_walk on 3 CTAs (many units and chunk switches per CTA: ring phases, restaging)
 #   tm_kb32   k_tm_walk with 32-kernel feature blocks (several blocks per CTA range)
 #   tm_ctas3  k_tm_walk on 3 CTAs (long per-CTA ranges crossing kernel blocks, many tasks/lane)
+#   tm_nsub3  k_tm_walk with every (kernel, tree) task split into 3 clock sub-ranges (uneven)
+#   tm_nsub64 k_tm_walk with 64 sub-ranges (single-clock sub-ranges on small tables)
 #   tm_slab   kernel slabs of 64 (several walk + finish launches reusing the zeroed D buffer)
 #   da        order-free difference-array kernel (k_sweep_da), shared-memory int64 sums
 #   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
@@ -50,6 +52,7 @@ DA = {"SYNERGY_ALGO": "da"}
 TR = {"SYNERGY_TM_MODE": "tr"}
 VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
             "tr_ctas3": {**TR, "SYNERGY_TR_CTAS": "3"}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
+            "tm_nsub3": {"SYNERGY_TM_NSUB": "3"}, "tm_nsub64": {"SYNERGY_TM_NSUB": "64"},
             "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
             "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
             "da_kpc5": {**DA, "SYNERGY_KPC": "5"}, "da_nsub3": {**DA, "SYNERGY_NSUB": "3"},
@@ -62,7 +65,7 @@ VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_TM_MODE", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+KNOBS = ("SYNERGY_TM_MODE", "SYNERGY_TM_NSUB", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
