@@ -74,6 +74,7 @@ struct TmArgs {
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
     int nsub;                    // clock sub-ranges per (kernel, tree) task (small batches)
+    int dyn;                     // k_tm_walk: tasks from a shared counter (small batches)
 };
 
 // One 2-level block step on clock-cut words (A = {thr(n), thr(c0), thr(c1), codes}, grandchild
@@ -107,6 +108,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
     float* xs = stk_c + kTmS * NT;                                           // [F + 2][NT] lane columns
     int* sroot = reinterpret_cast<int*>(xs + (size_t)(F + 2) * NT);         // [TT] root block per tree
+    __shared__ int s_next;                                                   // dynamic mode: next task offset
     int* const sb = stk_b + threadIdx.x;
     float* const sc = stk_c + threadIdx.x;
     float* const xcol = xs + threadIdx.x;
@@ -132,20 +134,28 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const int kbase = (int)(kbi * KB);                                   // slab-relative
         const int nvalid = min(KB, t.nks - kbase);
 
-        // Static lane streams: task j (tree j / KB, kernel-in-block j % KB) of the segment goes to
-        // lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same kernel kk and its
-        // trees advance by NT / KB: the lane's feature column is loaded once per segment.
+        // Static lane streams (large batches): task j (tree j / KB, kernel-in-block j % KB) of the
+        // segment goes to lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same
+        // kernel kk and its trees advance by NT / KB.  Dynamic (t.dyn, batches of a few tasks per
+        // lane): lanes take their first task by thread index and the next ones from a shared
+        // counter, so lanes that drew short walks take the remaining tasks; the lane's feature
+        // column is reloaded when its kernel changes.
         const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);
         int q;
-        {
+        if (t.dyn) {
+            __syncthreads();                                                 // previous segment's counter
+            if (threadIdx.x == 0) s_next = seg0 + NT;
+            __syncthreads();
+            q = seg0 + threadIdx.x;
+        } else {
             const int nw = NT / 32, w = threadIdx.x >> 5;
             const int g0 = seg0 >> 5;
             const int g = g0 + ((w - g0 % nw) + nw) % nw;
             q = 32 * g + lane;
             if (q < seg0) q += NT;
         }
-        const int kk = q & (KB - 1);
-        long long* const dbase = t.D + (size_t)(kbase + kk) * t.nslot * n_f;
+        int kk = -1;
+        long long* dbase = t.D;
         const uint4* blocks = a.ms.blocks;
         long long* drow = dbase;
         double scale = 1.0;
@@ -153,11 +163,23 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         int bk = 0, lo = 0, sn = 0, end = n_f;
         float tmin = CUDART_INF_F;
         long long vprev = 0;
-        bool active = kk < nvalid && q < seg1;
-        if (active) {
-            const float* g = a.features + (t.slab0 + kbase + kk) * F;
-            for (int c = 0; c < F; ++c) xcol[(size_t)c * NT] = __ldg(g + c);
-        }
+        bool active = false;
+        // take task offset q if it exists: its kernel's features into the lane column if new
+        auto take = [&](int qq) {
+            while (qq < seg1 && (qq & (KB - 1)) >= nvalid)                   // padding kernels
+                qq = t.dyn ? atomicAdd(&s_next, 1) : qq + NT;
+            q = qq;
+            active = qq < seg1;
+            if (!active) return;
+            const int k2 = qq & (KB - 1);
+            if (k2 != kk) {
+                kk = k2;
+                dbase = t.D + (size_t)(kbase + kk) * t.nslot * n_f;
+                const float* g = a.features + (t.slab0 + kbase + kk) * F;
+                for (int c = 0; c < F; ++c) xcol[(size_t)c * NT] = __ldg(g + c);
+            }
+        };
+        take(q);
         // start the task at offset q: tree (q / KB) / NS, clock sub-range (q / KB) % NS of this
         // lane's kernel.  A sub-range [lo, end) walks from the root at clock lo and, at its end,
         // takes its last value back out at D[end] so the difference arrays stay exact.
@@ -213,8 +235,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                 } else {
                     if (end < n_f)                                           // sub-range end: D[end] -= v
                         atomicAdd(reinterpret_cast<unsigned long long*>(drow + end), (unsigned long long)(-v));
-                    q += NT;                                                 // next task, same kernel
-                    active = q < seg1;
+                    take(t.dyn ? atomicAdd(&s_next, 1) : q + NT);            // next task
                     if (active) start(q);
                 }
             }

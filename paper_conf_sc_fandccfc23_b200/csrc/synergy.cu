@@ -634,6 +634,8 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         const int ns_env = env_int("SYNERGY_TM_NSUB", t.nsub);
         if (ns_env >= 1 && ns_env <= n_f && ns_env <= 64) t.nsub = ns_env;
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * t.nsub * kb;
+        // a few tasks per lane: dynamic task fetch balances walks of different lengths
+        t.dyn = env_int("SYNERGY_TM_DYN", t.n_tasks < 4 * lanes ? 1 : 0) ? 1 : 0;
         if (use_tr) {
             // unit = (tree, chunk of P kernels), one CTA per SM over contiguous unit ranges
             r.nchunks = (t.nks + P - 1) / P;
