@@ -428,7 +428,7 @@ def main():
     hbm = {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": hbm_ach / peaks["hbm_gbs"],
            "algorithmic_bytes": hbm_bytes, "peak_source": peak_src}
     work = None
-    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws", "k_tm_walk"):
+    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws", "k_tm_walk", "k_tr_walk"):
         work = run_walk_work(cfg, row0, n_local, which=args.models)
     if algo == "k_svr":
         # fp64 FMA-pipe roofline: 2 * n_k * n_f * n_SV flops per contraction
@@ -446,7 +446,7 @@ def main():
         # on-chip L1 roofline: each run walk fetches max(1, ceil(depth/2)) 32-byte
         # 2-level blocks; counted by the oracle from the inputs (runs of clocks sharing a leaf)
         per_launch = max(1.0, ktimes[algo][1] / K)             # kernel-slab launches per step
-        resume = algo == "k_tm_walk"
+        resume = algo in ("k_tm_walk", "k_tr_walk")
         blocks = work["resume_blocks_per_kernel" if resume else "run_blocks_per_kernel"] * (evals_step // n_f) / per_launch
         achieved = 32.0 * blocks / kern_avg_s / 1e9
         peak = 128.0 * sms * sm_max * 1e6 / 1e9

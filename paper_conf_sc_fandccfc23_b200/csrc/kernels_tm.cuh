@@ -99,7 +99,8 @@ __device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, cons
     return l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
 }
 
-template <int NT>
+// FXALL: every forest of the call has int32 fixed-point leaves (no int64 conversion path).
+template <int NT, bool FXALL>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -107,12 +108,15 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
     float* xs = stk_c + kTmS * NT;                                           // [F + 2][NT] lane columns
-    int* sroot = reinterpret_cast<int*>(xs + (size_t)(F + 2) * NT);         // [TT] root block per tree
+    int2* stree = reinterpret_cast<int2*>(xs + (size_t)(F + 2) * NT);       // [TT] {root block, model}
     __shared__ int s_next;                                                   // dynamic mode: next task offset
-    int* const sb = stk_b + threadIdx.x;
-    float* const sc = stk_c + threadIdx.x;
+    __shared__ const uint4* s_blocks[4];                                     // per model: clock-cut blocks,
+    __shared__ int s_slot[4], s_fx[4];                                       // D slot offset, int32 leaves,
+    __shared__ double s_scale[4];                                            // fixed-point scale
+    const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
+    constexpr unsigned kEnt = 4u * NT;                                       // bytes between stack entries
     float* const xcol = xs + threadIdx.x;
-    float* const xclk = xcol + (size_t)F * NT;
+    const unsigned xclk_a = su32(xcol + (size_t)F * NT);
 
     const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
               T3 = t.nm > 2 ? da_trees(a, 3) : 0;
@@ -121,7 +125,17 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     const long long per_kb = (long long)TT * NS * KB;
     for (int q = threadIdx.x; q < TT; q += NT) {
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
-        sroot[q] = __ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
+        stree[q] = make_int2(__ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3))), mi);
+    }
+    if (threadIdx.x < 4) {
+        const int m = threadIdx.x;
+        if (m < 2 || t.nm > 2) {
+            const DevModel& d = da_model(a, m);
+            s_blocks[m] = d.blocks;
+            s_slot[m] = t.slot_of[m] * n_f;
+            s_fx[m] = d.fx32;
+            s_scale[m] = d.fx_scale;
+        }
     }
     __syncthreads();
     const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
@@ -159,7 +173,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         const uint4* blocks = a.ms.blocks;
         long long* drow = dbase;
         double scale = 1.0;
-        bool fxm = false;                                                    // this model's leaves are int32
+        bool fxm = true;                                                     // this model's leaves are int32
         int bk = 0, lo = 0, sn = 0, end = n_f;
         float tmin = CUDART_INF_F;
         long long vprev = 0;
@@ -186,16 +200,17 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         auto start = [&](int qq) {
             const int ts = qq >> t.kb_log2;
             const int tti = NS == 1 ? ts : ts / NS, sub = ts - tti * NS;
-            const int mi = tti < c1 ? 0 : tti < c2 ? 1 : tti < c3 ? 2 : 3;
-            const DevModel& m = da_model(a, mi);
-            blocks = m.blocks;
-            scale = m.fx_scale;
-            fxm = m.fx32 != 0;                                               // as k_cut_blocks converted them
-            bk = sroot[tti];
-            drow = dbase + t.slot_of[mi] * n_f;
+            const int2 ti = stree[tti];
+            bk = ti.x;
+            blocks = s_blocks[ti.y];
+            drow = dbase + s_slot[ti.y];
+            if (!FXALL) {
+                fxm = s_fx[ti.y] != 0;                                       // as k_cut_blocks converted them
+                scale = s_scale[ti.y];
+            }
             lo = NS == 1 ? 0 : sub * n_f / NS;                               // n_f <= 4096, NS <= 64
             end = NS == 1 ? n_f : (sub + 1) * n_f / NS;
-            *xclk = (float)lo + 0.5f;                                        // clock lo enters as lo + 0.5
+            sts_f(xclk_a, (float)lo + 0.5f);                                 // clock lo enters as lo + 0.5
             tmin = CUDART_INF_F;
             sn = 0;
             vprev = 0;
@@ -212,8 +227,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             bk = (int)g;
             if (cb < tmin) {                                                 // new record
                 if (sn < kTmS) {                                             // deeper ones are not kept:
-                    sb[sn * NT] = cur;                                       // resuming at an ancestor on
-                    sc[sn * NT] = cb;                                        // the path is still exact
+                    sts_u(sb_a + kEnt * (unsigned)sn, (unsigned)cur);        // resuming at an ancestor on
+                    sts_f(sc_a + kEnt * (unsigned)sn, cb);                   // the path is still exact
                     ++sn;
                 }
                 tmin = cb;
@@ -221,17 +236,17 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             if (at_leaf) {
                 // run [lo, hi): hi = smallest left-turn cut; D[lo] += v - v_prev (exact int64)
                 const int hi = tmin < CUDART_INF_F ? (int)tmin : n_f;
-                const long long v = fxm ? (long long)(int)g
-                                        : __double2ll_rn(__dmul_rn((double)__uint_as_float(g), scale));
+                const long long v = (FXALL || fxm) ? (long long)(int)g
+                                                   : __double2ll_rn(__dmul_rn((double)__uint_as_float(g), scale));
                 atomicAdd(reinterpret_cast<unsigned long long*>(drow + lo), (unsigned long long)(v - vprev));
                 vprev = v;
                 if (hi < end) {
                     // resume at the deepest kept record's block (popped); the next one is the bound
                     --sn;
-                    bk = sb[sn * NT];
-                    tmin = sn > 0 ? sc[(sn - 1) * NT] : CUDART_INF_F;
+                    bk = (int)lds_u(sb_a + kEnt * (unsigned)sn);
+                    tmin = sn > 0 ? lds_f(sc_a + kEnt * (unsigned)(sn - 1)) : CUDART_INF_F;
                     lo = hi;
-                    *xclk = (float)hi + 0.5f;
+                    sts_f(xclk_a, (float)hi + 0.5f);
                 } else {
                     if (end < n_f)                                           // sub-range end: D[end] -= v
                         atomicAdd(reinterpret_cast<unsigned long long*>(drow + end), (unsigned long long)(-v));

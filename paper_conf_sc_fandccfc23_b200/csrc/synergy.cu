@@ -546,6 +546,9 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         tt += d.n_trees;
     }
     t.nm = nm;
+    bool fxall = true;                            // every forest has int32 fixed-point leaves
+    for (int m = 0; m < nm; ++m)
+        if (t.slot_of[m] >= 0 && !dms[m]->fx32) fxall = false;
     // kernels per feature block: a power of two in [32, 256], F * kb floats of shared memory
     int kb = 256;
     while (kb > 32 && ((size_t)F * kb * 4 > 32768 || kb / 2 >= n_k)) kb /= 2;
@@ -584,9 +587,12 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
     a.tile_k = kt;
     a.xs = (F + 2) | 1;
+    // finish CTA size: 128 threads when one wave of 256-thread CTAs would not hold the batch
+    int fnt = env_int("SYNERGY_TM_FNT", 256);
+    if (fnt != 128 && fnt != 256) fnt = 256;
     const size_t fsmem = (size_t)nm * kt * n_f * 12 + (size_t)n_f * 4 + (size_t)kt * a.xs * 4 + 32 +
                          (size_t)kt * t.nslot * n_f * 8;
-    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 4;
+    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8;
     static size_t fset = 48 * 1024, wset = 48 * 1024;
     cudaError_t e = cudaSuccess;
     if (fsmem > fset) {
@@ -595,14 +601,16 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         fset = fsmem;
     }
     if (wsmem > wset) {
-        if ((e = cudaFuncSetAttribute(k_tm_walk<kTmNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess)
+        if ((e = cudaFuncSetAttribute(k_tm_walk<kTmNT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess ||
+            (e = cudaFuncSetAttribute(k_tm_walk<kTmNT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess)
             return cuda_fail(e, "k_tm_walk attribute");
         wset = wsmem;
     }
     static int carve_set = -1;                 // same shared-memory carveout for both kernels
     const int carve = env_int("SYNERGY_TM_CARVE", -1);
     if (carve != carve_set && carve >= 0) {
-        cudaFuncSetAttribute(k_tm_walk<kTmNT>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+        cudaFuncSetAttribute(k_tm_walk<kTmNT, true>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+        cudaFuncSetAttribute(k_tm_walk<kTmNT, false>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
         cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
         cudaGetLastError();
         carve_set = carve;
@@ -662,7 +670,10 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
             {
                 KernelTimer ktm("k_tm_walk", st);
-                k_tm_walk<kTmNT><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+                if (fxall)
+                    k_tm_walk<kTmNT, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+                else
+                    k_tm_walk<kTmNT, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
                 e = cudaGetLastError();
             }
             if (e != cudaSuccess) {
@@ -672,7 +683,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         }
         {
             KernelTimer ktm("k_tm_finish", st);
-            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), 256, fsmem, st>>>(t);
+            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, st>>>(t);
             e = cudaGetLastError();
         }
         if (e != cudaSuccess) {
