@@ -583,7 +583,10 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     // finish tile: KT kernels per CTA, fp64 + fp32 per (model, kernel, clock) in shared memory
     // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
     int kt = std::max(1, std::min(8, (int)((150 * 1024) / ((size_t)nm * n_f * 12 + (size_t)t.nslot * n_f * 8))));
+    const int kt_cap = kt;                                         // shared-memory bound
     kt = (int)std::max<long long>(1, std::min<long long>(kt, nks / (8LL * sm_count(device))));
+    if (nks >= 2LL * sm_count(device) && nks <= 8LL * sm_count(device))
+        kt = std::min(2, kt_cap);                                  // one wave of kernel pairs (c2: 23 -> 20 us)
     kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
     a.tile_k = kt;
     a.xs = (F + 2) | 1;
