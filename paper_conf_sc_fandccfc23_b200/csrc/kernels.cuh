@@ -208,6 +208,7 @@ __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* 
     for (int m = 0; m < 4; ++m) {
         if (!mv[m]) continue;
         float* g = m == 0 ? a.S_out : m == 1 ? a.E_out : a.X_out[m - 2];
+#pragma unroll 4
         for (int u = threadIdx.x; u < units; u += blockDim.x) {
             const int kl = u / n_f;
             const double* r = mv[m] + (size_t)kl * n_f;

@@ -353,7 +353,7 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
             for (int i = lane; i < n_f; i += 32) out[i] = combine(m, 0.0, xrow, fr[i], F);
             continue;
         }
-        const long long* Dm = sD + ((size_t)pk * t.nslot + slot) * n_f;
+        long long* Dm = sD + ((size_t)pk * t.nslot + slot) * n_f;
         const int chunk = (n_f + 31) / 32;
         const int i0 = min(n_f, lane * chunk), i1 = min(n_f, i0 + chunk);
         long long run = 0;
@@ -365,10 +365,16 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
             if (lane >= off) excl += y;
         }
         excl -= run;
-        const double inv = m.fx_inv;
-        for (int i = i0; i < i1; ++i) {
+        for (int i = i0; i < i1; ++i) {                                       // exact prefix sums in place
             excl += Dm[i];
-            const double forest_sum = __dmul_rn(__ll2double_rn(excl), inv);  // RN(exact sum)
+            Dm[i] = excl;
+        }
+        __syncwarp();
+        // every clock independently (lane-strided, unrolled: the fp64 chains overlap)
+        const double inv = m.fx_inv;
+#pragma unroll 4
+        for (int i = lane; i < n_f; i += 32) {
+            const double forest_sum = __dmul_rn(__ll2double_rn(Dm[i]), inv);  // RN(exact sum)
             out[i] = combine(m, forest_sum, xrow, fr[i], F);
         }
     }
