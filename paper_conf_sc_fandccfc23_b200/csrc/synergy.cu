@@ -390,7 +390,7 @@ cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaS
 struct TmBuf {
     int dev;
     cudaStream_t st;
-    int kind;                        // 0: D (kept all-zero between calls), 1: k_tr_walk features
+    int kind;                        // 0/2: D and its second slab buffer (all-zero between calls), 1: k_tr_walk features
     long long* p;
     size_t bytes;
     bool dirty;
@@ -424,11 +424,43 @@ syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out, int ki
         b->bytes = bytes;
         b->dirty = true;
     }
-    if (b->dirty && kind == 0) {
+    if (b->dirty && kind != 1) {
         if ((e = cudaMemsetAsync(b->p, 0, b->bytes, st)) != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(D)");
         b->dirty = false;
     }
     *out = b;
+    return ok();
+}
+
+// Slab pipeline (several kernel slabs per call): the finish of slab i runs on a library-owned
+// second stream while the walk of slab i + 1 runs on the caller's stream, with D double-buffered.
+// One side stream and three events per (device, caller stream).
+struct TmAux {
+    int dev;
+    cudaStream_t st;
+    cudaStream_t st2;
+    cudaEvent_t walked[2], finished[2];
+};
+std::list<TmAux> g_tm_aux;
+
+syn_status tm_aux(int dev, cudaStream_t st, TmAux** out) {
+    std::lock_guard<std::mutex> lock(g_tm_mu);
+    for (TmAux& x : g_tm_aux)
+        if (x.dev == dev && x.st == st) {
+            *out = &x;
+            return ok();
+        }
+    TmAux x;
+    x.dev = dev;
+    x.st = st;
+    cudaError_t e = cudaStreamCreateWithFlags(&x.st2, cudaStreamNonBlocking);
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+        if ((e = cudaEventCreateWithFlags(&x.walked[i], cudaEventDisableTiming)) == cudaSuccess)
+            e = cudaEventCreateWithFlags(&x.finished[i], cudaEventDisableTiming);
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "slab pipeline stream/events");
+    g_tm_aux.push_back(x);
+    *out = &g_tm_aux.back();
     return ok();
 }
 
@@ -575,6 +607,15 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     syn_status s = tm_buffer(device, st, (size_t)nks * row, &buf);
     if (s != SYN_OK) return s;
     t.D = buf->p;
+    // several slabs: finish(i) on a side stream overlaps walk(i + 1); D alternates between two
+    // buffers and walk(i + 2) waits for finish(i), which zeroes its buffer
+    const bool pipe = n_k > nks && env_int("SYNERGY_TM_PIPE", 1) != 0;
+    TmBuf* buf2 = nullptr;
+    TmAux* aux = nullptr;
+    if (pipe) {
+        if ((s = tm_buffer(device, st, (size_t)nks * row, &buf2, 2)) != SYN_OK) return s;
+        if ((s = tm_aux(device, st, &aux)) != SYN_OK) return s;
+    }
     if (use_tr && F > 0) {
         TmBuf* fb = nullptr;
         if ((s = tm_buffer(device, st, (size_t)((nks + P - 1) / P) * F * P * 4, &fb, 1)) != SYN_OK) return s;
@@ -633,9 +674,16 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     }
     t.s = a;
     int n = 0;
-    for (long long s0 = 0; s0 < n_k; s0 += nks) {
+    int slab = 0;
+    for (long long s0 = 0; s0 < n_k; s0 += nks, ++slab) {
         t.slab0 = s0;
         t.nks = (int)std::min<long long>(nks, n_k - s0);
+        const int pb = slab & 1;
+        if (pipe) {
+            t.D = pb ? buf2->p : buf->p;
+            if (slab >= 2 && (e = cudaStreamWaitEvent(st, aux->finished[pb], 0)) != cudaSuccess)
+                return cuda_fail(e, "slab pipeline wait");
+        }
         // tiny batches: split every (kernel, tree) task into clock sub-ranges while there are fewer
         // tasks than resident lanes (at most 8 sub-ranges of at least 8 clocks; each sub-range
         // adds a root descent, so batches with a task per lane keep whole tasks)
@@ -666,6 +714,8 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             }
             if (e != cudaSuccess) {
                 buf->dirty = true;
+                if (buf2) buf2->dirty = true;
+                if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
                 return cuda_fail(e, "k_tr_walk launch");
             }
             ++n;
@@ -681,20 +731,36 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             }
             if (e != cudaSuccess) {
                 buf->dirty = true;
+                if (buf2) buf2->dirty = true;
+                if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
                 return cuda_fail(e, "k_tm_walk launch");
             }
         }
+        cudaStream_t fst = st;
+        if (pipe) {
+            if ((e = cudaEventRecord(aux->walked[pb], st)) != cudaSuccess ||
+                (e = cudaStreamWaitEvent(aux->st2, aux->walked[pb], 0)) != cudaSuccess) {
+                buf->dirty = buf2->dirty = true;
+                return cuda_fail(e, "slab pipeline fork");
+            }
+            fst = aux->st2;
+        }
         {
-            KernelTimer ktm("k_tm_finish", st);
-            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, st>>>(t);
+            KernelTimer ktm("k_tm_finish", fst);
+            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, fst>>>(t);
             e = cudaGetLastError();
         }
+        if (e == cudaSuccess && pipe) e = cudaEventRecord(aux->finished[pb], aux->st2);
         if (e != cudaSuccess) {
             buf->dirty = true;
+            if (buf2) buf2->dirty = true;
+            if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
             return cuda_fail(e, "k_tm_finish launch");
         }
         n += 2;
     }
+    if (pipe && (e = cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0)) != cudaSuccess)   // join
+        return cuda_fail(e, "slab pipeline join");
     *launches = n;
     *variant = use_tr ? 4001 : 4000;
     return ok();
