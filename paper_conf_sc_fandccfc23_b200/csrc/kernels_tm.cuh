@@ -41,7 +41,7 @@
 //
 //  * Accumulation in L2.  Run j of a (kernel, model, tree) adds v_j - v_{j-1} to
 //    D[kernel][slot][lo_j] with one 64-bit global reduction (exact, order-free; run 0 adds v_0).
-//    No shared-memory difference arrays: shared memory stays ~15 KB per CTA so L1 keeps the
+//    No shared-memory difference arrays: shared memory stays ~54 KB per CTA so L1 keeps the
 //    trees.  k_tm_finish then scans each D row (exact int64 prefix sum = the exact leaf sum per
 //    clock), rounds it once, combines the members and runs finish_tile4; it zeroes D as it reads
 //    it, so the next call starts from zeros without a memset.
