@@ -1,0 +1,87 @@
+"""The fused path on several streams at once and inside a CUDA graph (DESIGN.md §6 slab pipeline:
+library-owned difference-array buffers and side stream per (device, caller stream); the side
+stream forks from and joins the caller's stream with events, so a captured call is a fork-join
+graph).  Results are compared with the CPU oracle, bit for bit."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_sc_fandccfc23_b200 import workloads as W
+from gpu_util import assert_bits_equal
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _build():
+    from paper_conf_sc_fandccfc23_b200 import build
+    build.build()
+    oracle.build()
+
+
+def _workload(seed):
+    # several kernel slabs at SYNERGY_TM_SLAB=64: the pipeline runs (finish i || walk i + 1)
+    return W.fuzz_workload(seed, 300, 64, F=5, n_trees=4, max_depth=8, p_leaf=0.1)
+
+
+def _run(w, stream, S, E, out):
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    sp, en, ck = syn.Model(w.speedup), syn.Model(w.energy), syn.Clocks(w.freqs)
+    feats = torch.from_numpy(np.ascontiguousarray(w.features)).cuda()
+    return (sp, en, ck, feats), lambda: syn.sweep(sp, en, feats, ck, w.default_idx, w.targets, out=out,
+                                                  out_speedup=S, out_energy=E, stream=stream)
+
+
+def _buffers(w):
+    import torch
+    S = torch.full((w.n_kernels, w.n_freqs), -1.0, dtype=torch.float32, device="cuda")
+    E = torch.full_like(S, -1.0)
+    out = torch.full((w.n_kernels, len(w.targets)), -9, dtype=torch.int32, device="cuda")
+    return S, E, out
+
+
+def _check(w, S, E, out):
+    ref = oracle.sweep_workload(w, want_pred=True)
+    assert_bits_equal(S.cpu().numpy(), ref["S"], "S")
+    assert_bits_equal(E.cpu().numpy(), ref["E"], "E")
+    assert np.array_equal(out.cpu().numpy(), ref["choice"])
+
+
+def test_two_streams_concurrently(monkeypatch):
+    import torch
+    monkeypatch.setenv("SYNERGY_TM_SLAB", "64")
+    monkeypatch.setenv("SYNERGY_TM_KB", "32")
+    ws = [_workload(5), _workload(6)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    bufs = [_buffers(w) for w in ws]
+    runs = [_run(w, s.cuda_stream, *b) for w, s, b in zip(ws, streams, bufs)]
+    torch.cuda.synchronize()
+    for _ in range(3):                                   # interleaved calls on both streams
+        for (_, call), s in zip(runs, streams):
+            with torch.cuda.stream(s):
+                call()
+    torch.cuda.synchronize()
+    for w, b in zip(ws, bufs):
+        _check(w, *b)
+
+
+def test_captured_in_cuda_graph(monkeypatch):
+    import torch
+    monkeypatch.setenv("SYNERGY_TM_SLAB", "64")
+    monkeypatch.setenv("SYNERGY_TM_KB", "32")
+    w = _workload(7)
+    S, E, out = _buffers(w)
+    s = torch.cuda.Stream()
+    keep, call = _run(w, s.cuda_stream, S, E, out)
+    with torch.cuda.stream(s):
+        call()                                           # warm-up: builds the cached buffers
+    torch.cuda.synchronize()
+    S.fill_(-1.0); E.fill_(-1.0); out.fill_(-9)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        call()
+    for _ in range(3):
+        g.replay()
+    torch.cuda.synchronize()
+    _check(w, S, E, out)
