@@ -24,8 +24,15 @@
  *     stream).  Results are valid after the caller synchronises that stream.  Launch failures
  *     return SYN_ERR_CUDA.
  *   - "d_" pointers are device pointers on the model's device, "h_" pointers host pointers.
- *     The caller owns every buffer it passes; the hot calls never allocate, except the
- *     stream-ordered SVR scratch described at syn_model_desc.
+ *     The caller owns every buffer it passes.  The library keeps its own scratch, created on
+ *     first use and reused afterwards: per (model, clock table) a clock-cut copy of the forest
+ *     (built synchronously by the first call that pairs them); per (device, stream) the
+ *     int64 difference arrays of the sweep (grown on demand, SYN_ERR_OOM possible), and for
+ *     calls spanning several kernel slabs a second array, a side stream and events (the
+ *     finish of slab i overlaps the walk of slab i + 1; the call joins the side stream before
+ *     returning); and the stream-ordered SVR scratch described at syn_model_desc.  After one
+ *     call of a given shape on a stream, later such calls only enqueue work, so they may be
+ *     captured into a CUDA graph.
  *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
  *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
  *   - Handles (models, clock tables, workspaces) are bound to the device they were created
