@@ -104,6 +104,7 @@ template <int NT, bool FXALL>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
     extern __shared__ __align__(16) unsigned char smem[];
+    asm volatile("griddepcontrol.launch_dependents;");                       // k_tm_finish may launch early
     const int n_f = a.n_f, F = a.F, KB = t.kb;
     int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
@@ -334,6 +335,9 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
         xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
     }
     for (int i = threadIdx.x; i < n_f; i += blockDim.x) fr[i] = __ldg(a.freqs + i);
+    // launched as a programmatic dependent of k_tm_walk (same stream): everything above overlaps
+    // the walk's tail; D is read only after the walk grid has completed (no-op otherwise)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     // this CTA's D rows are one contiguous region: stage it with independent coalesced loads,
     // then zero it for the next call
     long long* gD = t.D + (size_t)k0s * t.nslot * n_f;

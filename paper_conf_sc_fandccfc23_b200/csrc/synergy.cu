@@ -747,8 +747,25 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         }
         {
             KernelTimer ktm("k_tm_finish", fst);
-            k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, fst>>>(t);
-            e = cudaGetLastError();
+            if (!pipe && env_int("SYNERGY_TM_PDL", 1) != 0) {
+                // programmatic dependent launch: the finish grid is scheduled while the walk runs
+                // and waits (griddepcontrol.wait) for it before reading D
+                cudaLaunchConfig_t lc;
+                memset(&lc, 0, sizeof lc);
+                lc.gridDim = dim3((unsigned)((t.nks + kt - 1) / kt));
+                lc.blockDim = dim3((unsigned)fnt);
+                lc.dynamicSmemBytes = fsmem;
+                lc.stream = fst;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+                at[0].val.programmaticStreamSerializationAllowed = 1;
+                lc.attrs = at;
+                lc.numAttrs = 1;
+                e = cudaLaunchKernelEx(&lc, k_tm_finish, t);
+            } else {
+                k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, fst>>>(t);
+                e = cudaGetLastError();
+            }
         }
         if (e == cudaSuccess && pipe) e = cudaEventRecord(aux->finished[pb], aux->st2);
         if (e != cudaSuccess) {

@@ -33,6 +33,7 @@ def _build():
 #   tm_nsub64 k_tm_walk with 64 sub-ranges (single-clock sub-ranges on small tables)
 #   tm_dyn    k_tm_walk with dynamic task fetch forced on (large batches: lanes change kernels)
 #   tm_static k_tm_walk with static lane streams forced on (small batches)
+#   tm_nopdl  k_tm_finish launched without programmatic dependent launch
 #   tm_slab   kernel slabs of 64 (several walk + finish launches; finish(i) on the side stream
 #             overlapping walk(i + 1), D double-buffered and re-zeroed by the finishes)
 #   tm_slab_seq  kernel slabs of 64 run in order on the caller's stream (one D buffer)
@@ -58,6 +59,7 @@ VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
             "tr_ctas3": {**TR, "SYNERGY_TR_CTAS": "3"}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
             "tm_nsub3": {"SYNERGY_TM_NSUB": "3"}, "tm_nsub64": {"SYNERGY_TM_NSUB": "64"},
             "tm_dyn": {"SYNERGY_TM_DYN": "1"}, "tm_static": {"SYNERGY_TM_DYN": "0"},
+            "tm_nopdl": {"SYNERGY_TM_PDL": "0"},
             "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
             "tm_slab_seq": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32", "SYNERGY_TM_PIPE": "0"},
             "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
@@ -71,7 +73,7 @@ VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
             "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
             "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
             "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_TM_PIPE", "SYNERGY_TM_DYN", "SYNERGY_TM_MODE", "SYNERGY_TM_NSUB", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+KNOBS = ("SYNERGY_TM_PDL", "SYNERGY_TM_PIPE", "SYNERGY_TM_DYN", "SYNERGY_TM_MODE", "SYNERGY_TM_NSUB", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
 
 
 @pytest.fixture(params=list(VARIANTS))
