@@ -217,8 +217,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             vprev = 0;
         };
         if (active) start(q);
-        while (__any_sync(0xffffffffu, active)) {
-            if (!active) continue;
+        while (active) {                                                     // lanes leave as they finish
             uint4 A, B;
             const int cur = bk;
             ldg_blk256(blocks + 2 * (size_t)cur, A, B);
