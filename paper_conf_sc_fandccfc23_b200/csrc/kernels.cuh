@@ -220,14 +220,23 @@ __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* 
     }
     if (a.mode != kModeSweep) return;
     __syncthreads();
-    const int n_t = a.n_t;
-    for (int task = threadIdx.x >> 5; task < nk * n_t; task += nw) {
+    // each warp takes a contiguous run of (row, target) tasks, so a row's baselines are computed
+    // once per warp that touches it instead of once per target
+    const int n_t = a.n_t, ntask = nk * n_t, per = (ntask + nw - 1) / nw;
+    const int tb = (threadIdx.x >> 5) * per, te = min(ntask, tb + per);
+    int row = -1;
+    bool base_ok = false;
+    double E_def = 0.0, S_def = 0.0, E_min = 0.0, S_minE = 0.0;
+    for (int task = tb; task < te; ++task) {
         const int kl = task / n_t, t = task - kl * n_t;
         const float* S = sv[0] + (size_t)kl * n_f;
         const float* E = sv[1] + (size_t)kl * n_f;
-        double E_def, S_def, E_min, S_minE;
+        if (kl != row) {
+            row = kl;
+            base_ok = select_baseline(S, E, n_f, a.def, lane, E_def, S_def, E_min, S_minE);
+        }
         int c = -1;
-        if (select_baseline(S, E, n_f, a.def, lane, E_def, S_def, E_min, S_minE))
+        if (base_ok)
             c = select_target(S, E, mv[2] ? sv[2] + (size_t)kl * n_f : nullptr,
                               mv[3] ? sv[3] + (size_t)kl * n_f : nullptr, n_f, a.kind[t], a.x[t],
                               E_def, S_def, E_min, S_minE, lane);
