@@ -625,20 +625,39 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
     int kt = std::max(1, std::min(8, (int)((150 * 1024) / ((size_t)nm * n_f * 12 + (size_t)t.nslot * n_f * 8))));
     const int kt_cap = kt;                                         // shared-memory bound
-    kt = (int)std::max<long long>(1, std::min<long long>(kt, nks / (8LL * sm_count(device))));
-    if (nks >= 2LL * sm_count(device) && nks <= 8LL * sm_count(device))
-        kt = std::min(2, kt_cap);                                  // one wave of kernel pairs (c2: 23 -> 20 us)
-    kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
-    a.tile_k = kt;
     a.xs = (F + 2) | 1;
-    // finish CTA size: 128 threads when one wave of 256-thread CTAs would not hold the batch
-    int fnt = env_int("SYNERGY_TM_FNT", 256);
+    int fnt = env_int("SYNERGY_TM_FNT", 256);                     // finish CTA size
     if (fnt != 128 && fnt != 256) fnt = 256;
-    const size_t fsmem = (size_t)nm * kt * n_f * 12 + (size_t)n_f * 4 + (size_t)kt * a.xs * 4 + 32 +
-                         (size_t)kt * t.nslot * n_f * 8;
-    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8;
+    auto fsmem_of = [&](int k) {
+        return (size_t)nm * k * n_f * 12 + (size_t)n_f * 4 + (size_t)k * a.xs * 4 + 32 + (size_t)k * t.nslot * n_f * 8;
+    };
     static size_t fset = 48 * 1024, wset = 48 * 1024;
     cudaError_t e = cudaSuccess;
+    if (fsmem_of(kt_cap) > fset) {
+        if ((e = cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem_of(kt_cap))) != cudaSuccess)
+            return cuda_fail(e, "k_tm_finish attribute");
+        fset = fsmem_of(kt_cap);
+    }
+    // the smallest tile whose finish grid fits in one wave of resident CTAs (a partial second wave
+    // doubles the finish's latency chain: c5 KT 3 -> 7 = 1195 -> 512 CTAs, 46 -> 37 us); when no
+    // tile fits, the largest (kt_cap)
+    {
+        const int sms = sm_count(device);
+        int fit = 0;
+        for (int k = 1; k <= kt_cap && !fit; ++k) {
+            int nb = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tm_finish, fnt, fsmem_of(k)) != cudaSuccess) {
+                cudaGetLastError();
+                break;
+            }
+            if (nb > 0 && (nks + k - 1) / k <= (long long)nb * sms) fit = k;
+        }
+        kt = fit ? fit : kt_cap;
+    }
+    kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
+    a.tile_k = kt;
+    const size_t fsmem = fsmem_of(kt);
+    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8;
     if (fsmem > fset) {
         if ((e = cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem)) != cudaSuccess)
             return cuda_fail(e, "k_tm_finish attribute");
