@@ -212,10 +212,10 @@ def oracle_single_core(cfg, n_k_cap, budget_s=10.0, which="rf"):
 
 
 def run_walk_work(cfg, row0, n_rows, budget=5e8, which="rf"):
-    """Run-walk work of the launched rows, counted by the oracle on the first rows that fit a
-    budget of ~5e8 node decisions (all rows for c1/c2/c5): runs of clocks sharing a leaf and their
-    2-level block fetches."""
-    import oracle
+    """Run-walk work of the launched rows, counted by the measurement tool tools/workcount.c (not
+    the oracle) on the first rows that fit a budget of ~5e8 node decisions (all rows for c1/c2/c5):
+    runs of clocks sharing a leaf and their 2-level block fetches."""
+    import tools
     from paper_conf_sc_fandccfc23_b200 import workloads as W
     n_f = W.CONFIGS[cfg][1]
     models = bench_models(cfg, which)
@@ -225,7 +225,7 @@ def run_walk_work(cfg, row0, n_rows, budget=5e8, which="rf"):
     if n == 0:
         return None
     w = W.make_config(cfg, row0=row0, n=n, models=models)
-    r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
+    r = tools.count([w.speedup, w.energy], w.features, w.freqs)
     trees = w.speedup.n_trees + w.energy.n_trees
     return {"run_blocks_per_kernel": r["run_blocks"] / n, "resume_blocks_per_kernel": r["resume_blocks"] / n,
             "runs_per_kernel_tree": r["runs"] / (n * max(trees, 1)),

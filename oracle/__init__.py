@@ -67,9 +67,6 @@ def _load():
         lib.oracle_sweep4.restype = C.c_int
         lib.oracle_sweep4.argtypes = [P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32, P, P,
                                       C.c_int32, P, P]
-        lib.oracle_sweep_stats.restype = C.c_int
-        lib.oracle_sweep_stats.argtypes = [P, P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32,
-                                           P, P, C.c_int32, P, P, P, P, P, P]
         lib.oracle_sweep.restype = C.c_int
         lib.oracle_sweep.argtypes = [P, P, P, C.c_int64, C.c_int32, P, C.c_int32, C.c_int32,
                                      P, P, C.c_int32, P, P, P, P, P]
@@ -190,27 +187,6 @@ def sweep(speedup, energy, features, freqs, default_idx, targets, want_pred=Fals
     if count_visits:
         out["visits"] = int(v[0])
     return out
-
-
-def sweep_stats(speedup, energy, features, freqs, default_idx, targets):
-    """Choices plus the run-walk work counters (visits, runs, run_decisions, run_blocks,
-    resume_blocks)."""
-    lib = _load()
-    ks, ke = _Keep(speedup), _Keep(energy)
-    features = np.ascontiguousarray(features, dtype=np.float32)
-    freqs = np.ascontiguousarray(freqs, dtype=np.float32)
-    n_k, F = features.shape
-    kinds, xs = _targets(targets)
-    ch = np.empty((n_k, len(kinds)), np.int32)
-    c = np.zeros(5, np.int64)
-    rc = lib.oracle_sweep_stats(ks.ref, ke.ref, _ptr(features), n_k, F, _ptr(freqs), freqs.shape[0],
-                                int(default_idx), _ptr(kinds), _ptr(xs), len(kinds), _ptr(ch),
-                                c[0:].ctypes.data, c[1:].ctypes.data, c[2:].ctypes.data, c[3:].ctypes.data,
-                                c[4:].ctypes.data)
-    if rc != 0:
-        raise OracleError("oracle_sweep_stats: invalid arguments")
-    return {"choice": ch, "visits": int(c[0]), "runs": int(c[1]), "run_decisions": int(c[2]),
-            "run_blocks": int(c[3]), "resume_blocks": int(c[4])}
 
 
 def sweep4(models, features, freqs, default_idx, targets, want_pred=False):

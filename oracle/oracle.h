@@ -11,6 +11,7 @@
  *   EDP = e*t, ED2P = e*t^2                                          L253 (§5.1)
  *   ES_x (x% of the potential saving vs default; ES_100 = min energy) L259-L267 (§5.2)
  *   PL_x (x% of the potential performance loss, same interval)        L269-L271 (§5.3)
+ *   absolute-saving reading "best performance with x% energy savings"  L11, L46 (§1)
  *   model families Linear / RandomForest                              L386, Table 2
  * Readings of silent/ambiguous points: DESIGN.md "Readings" (Q1..Q23 of SURVEY §8(c)).
  * Compile: gcc -O2 -std=c99 -ffp-contract=off (no fast-math).
@@ -56,8 +57,9 @@ int oracle_predict(const oracle_model *speedup, const oracle_model *energy,
                    const float *freqs, int32_t n_f, int32_t default_idx,
                    float *S, float *E, int64_t *visits);
 
-/* choice[k][t] for targets (kind[t], x[t]); kinds 0..5 = MAX_PERF, MIN_ENERGY, MIN_EDP,
- * MIN_ED2P, ES, PL.  gap (nullable) [n_k][n_t] receives the relative gap between the best
+/* choice[k][t] for targets (kind[t], x[t]); kinds 0..7 = MAX_PERF, MIN_ENERGY, MIN_EDP,
+ * MIN_ED2P, ES, PL (potential-saving reading, L267/L271), ES_ABS, PL_ABS (absolute reading
+ * E <= (1-x%) E_def resp. S >= (1-x%) S_def, L11/L46; -1 when no clock qualifies).  gap (nullable) [n_k][n_t] receives the relative gap between the best
  * and the runner-up key among feasible candidates (+inf if fewer than two). */
 int oracle_select(const float *S, const float *E, int64_t n_k, int32_t n_f,
                   int32_t default_idx, const int32_t *kind, const float *x, int32_t n_t,
@@ -69,18 +71,6 @@ int oracle_sweep(const oracle_model *speedup, const oracle_model *energy,
                  const float *freqs, int32_t n_f, int32_t default_idx,
                  const int32_t *kind, const float *x, int32_t n_t,
                  int32_t *choice, float *S, float *E, double *gap, int64_t *visits);
-
-/* oracle_sweep plus work counters of the run-walk algorithm (DESIGN.md §6 roofline): runs =
- * maximal clock runs sharing a leaf per (kernel, tree), run_decisions = sum of their leaf depths,
- * run_blocks = sum of max(1, ceil(depth/2)), resume_blocks = block fetches when every run after
- * the first resumes at the block where its path leaves the previous run's (kernels_tm.cuh).
- * Counters are added to (not reset). */
-int oracle_sweep_stats(const oracle_model *speedup, const oracle_model *energy,
-                       const float *features, int64_t n_k, int32_t n_features,
-                       const float *freqs, int32_t n_f, int32_t default_idx,
-                       const int32_t *kind, const float *x, int32_t n_t,
-                       int32_t *choice, int64_t *visits, int64_t *runs, int64_t *run_decisions,
-                       int64_t *run_blocks, int64_t *resume_blocks);
 
 /* Four-model variant: models[0] speedup, [1] energy, [2] EDP, [3] ED2P
  * ([2]/[3] nullable = derived).  MIN_EDP / MIN_ED2P use the direct model's normalised

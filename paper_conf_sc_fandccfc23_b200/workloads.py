@@ -28,9 +28,10 @@ from typing import Optional
 import numpy as np
 
 # Energy-target kinds (include/synergy.h: syn_target_kind).  PAPER L182, L382, Table 2.
-MAX_PERF, MIN_ENERGY, MIN_EDP, MIN_ED2P, ES, PL = 0, 1, 2, 3, 4, 5
+# ES_ABS / PL_ABS: the absolute-saving reading of L11/L46 (Q1).
+MAX_PERF, MIN_ENERGY, MIN_EDP, MIN_ED2P, ES, PL, ES_ABS, PL_ABS = 0, 1, 2, 3, 4, 5, 6, 7
 TARGET_NAMES = {MAX_PERF: "MAX_PERF", MIN_ENERGY: "MIN_ENERGY", MIN_EDP: "MIN_EDP",
-                MIN_ED2P: "MIN_ED2P", ES: "ES", PL: "PL"}
+                MIN_ED2P: "MIN_ED2P", ES: "ES", PL: "PL", ES_ABS: "ES_ABS", PL_ABS: "PL_ABS"}
 
 N_STATIC = 12           # Table 1's ten counts + two synthetic count columns
 SEED_BASE = 0x5EED0000

@@ -121,3 +121,9 @@ def test_choice_error_exact_rationals_and_missing():
             apes.append(a)
         assert cnt[t] == len(apes)
         assert abs(mape[t] - float(sum(apes) / len(apes))) < 1e-14
+        # RMSE over the counted kernels (L388-L392): sqrt(mean of (pred - actual)^2), exact rationals.
+        # Some predictions are -1 (not counted), so normalising by n_k instead would fail here.
+        ms = sum((obj(k, pred[k, t]) - obj(k, truth[k, t])) ** 2 for k in range(n_k) if pred[k, t] >= 0) / len(apes)
+        assert len(apes) < n_k
+        assert abs(Fraction(rmse[t]) ** 2 - ms) <= Fraction(1, 10 ** 14) * max(ms, Fraction(1, 10 ** 6))
+        assert ms > 0

@@ -13,8 +13,8 @@ from fractions import Fraction
 import numpy as np
 import pytest
 
-from paper_conf_sc_fandccfc23_b200.workloads import (ES, MAX_PERF, MIN_ED2P, MIN_EDP, MIN_ENERGY,
-                                                     PL, TARGET_NAMES)
+from paper_conf_sc_fandccfc23_b200.workloads import (ES, ES_ABS, MAX_PERF, MIN_ED2P, MIN_EDP, MIN_ENERGY,
+                                                     PL, PL_ABS, TARGET_NAMES)
 
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 KIND = {v: k for k, v in TARGET_NAMES.items()}
@@ -30,7 +30,7 @@ def _load_golden(name):
     return S, E, g["default_idx"], targets, expected
 
 
-@pytest.mark.parametrize("name", ["worked_example.json", "non_pareto_default.json"])
+@pytest.mark.parametrize("name", ["worked_example.json", "non_pareto_default.json", "absolute_targets.json"])
 def test_golden_examples(oracle_lib, name):
     S, E, d, targets, expected = _load_golden(name)
     ch = oracle_lib.select(S, E, d, targets)
@@ -72,6 +72,12 @@ def _brute(S, E, d, targets):
             elif kind == PL:
                 if s[i] >= s[d] - fr * (s[d] - s[i_min]):
                     cand.append((e[i], i))
+            elif kind == ES_ABS:                             # L11/L46, Q1
+                if e[i] <= (1 - fr) * e[d]:
+                    cand.append((-s[i], i))
+            elif kind == PL_ABS:
+                if s[i] >= (1 - fr) * s[d]:
+                    cand.append((e[i], i))
         out.append(min(cand)[1] if cand else -1)
     return out
 
@@ -93,6 +99,11 @@ ALL_TARGETS = [(MAX_PERF, 0.0), (MIN_ENERGY, 0.0), (MIN_EDP, 0.0), (MIN_ED2P, 0.
     [(ES, x) for x in (0.0, 25.0, 50.0, 75.0, 100.0)] + [(PL, x) for x in (0.0, 25.0, 50.0, 75.0, 100.0)]
 
 
+# absolute-saving targets with x whose x/100 and 1 - x/100 are exact dyadic fractions
+ABS_TARGETS = [(ES_ABS, x) for x in (0.0, 12.5, 25.0, 50.0, 75.0, 100.0)] + \
+    [(PL_ABS, x) for x in (0.0, 25.0, 50.0, 87.5, 100.0)] + [(ES, 37.5), (PL, 62.5)]
+
+
 def test_rational_brute_force_with_ties(oracle_lib):
     rng = np.random.default_rng(1234)
     n_cases = 10_000
@@ -100,8 +111,9 @@ def test_rational_brute_force_with_ties(oracle_lib):
         n = int(rng.integers(1, 9))
         S, E = _grid_case(rng, n)
         d = int(rng.integers(0, n))
-        ch = oracle_lib.select(S, E, d, ALL_TARGETS)[0].tolist()
-        assert ch == _brute(S, E, d, ALL_TARGETS), (c, S, E, d)
+        for tg in (ALL_TARGETS, ABS_TARGETS):
+            ch = oracle_lib.select(S, E, d, tg)[0].tolist()
+            assert ch == _brute(S, E, d, tg), (c, S, E, d)
 
 
 # ------------------------------------------------------------- Pareto-front formulation
@@ -241,7 +253,9 @@ def test_validation(oracle_lib):
     with pytest.raises(oracle_lib.OracleError):
         oracle_lib.select(S, S, 0, [(ES, 101.0)])          # x outside [0, 100]
     with pytest.raises(oracle_lib.OracleError):
-        oracle_lib.select(S, S, 0, [(7, 0.0)])             # unknown kind
+        oracle_lib.select(S, S, 0, [(8, 0.0)])             # unknown kind
+    with pytest.raises(oracle_lib.OracleError):
+        oracle_lib.select(S, S, 0, [(ES_ABS, -1.0)])       # x outside [0, 100]
     with pytest.raises(oracle_lib.OracleError):
         oracle_lib.select(S, S, 0, [(ES, float("nan"))])
     with pytest.raises(oracle_lib.OracleError):

@@ -1,5 +1,5 @@
-"""Pins for the oracle's run-walk work counters (oracle.c: oracle_sweep_stats), the numerator of
-the k_sweep_da roofline.  Checked against an independent formulation: a depth-first
+"""Pins for the run-walk work counters (tools/workcount.c, a measurement tool separate from the
+oracle), the numerator of the k_tm_walk roofline.  Checked against an independent formulation: a depth-first
 walk of each tree over the clock-index interval that splits at clock thresholds (each leaf reached
 owns one run of consecutive clocks), written here from the tree definition."""
 import numpy as np
@@ -43,8 +43,8 @@ def interval_runs(spec, t, x_static, freqs):
 
 
 def _check(w):
-    import oracle
-    r = oracle.sweep_stats(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets)
+    import tools
+    r = tools.count([w.speedup, w.energy], w.features, w.freqs)
     runs = dec = blk = res = 0
     for k in range(w.n_kernels):
         for m in (w.speedup, w.energy):
@@ -58,11 +58,18 @@ def _check(w):
                 res += e
     assert (r["runs"], r["run_decisions"], r["run_blocks"]) == (runs, dec, blk)
     assert r["resume_blocks"] == res
-    np.testing.assert_array_equal(r["choice"], oracle.sweep_workload(w)["choice"])
 
 
 def test_workcount_c1():
     _check(W.make_config("c1"))
+
+
+def test_decisions_are_t_times_d_on_complete_trees():
+    """Direct traversal of complete depth-D trees takes exactly T*D decisions per evaluation."""
+    import tools
+    w = W.make_config("c1")
+    r = tools.count([w.speedup, w.energy], w.features, w.freqs)
+    assert r["decisions"] == w.n_kernels * w.n_freqs * 2 * 10 * 8
 
 
 def test_workcount_fuzz_unbalanced_exact_thresholds():
