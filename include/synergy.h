@@ -24,15 +24,24 @@
  *     stream).  Results are valid after the caller synchronises that stream.  Launch failures
  *     return SYN_ERR_CUDA.
  *   - "d_" pointers are device pointers on the model's device, "h_" pointers host pointers.
- *     The caller owns every buffer it passes.  The library keeps its own scratch, created on
- *     first use and reused afterwards: per (model, clock table) a clock-cut copy of the forest
- *     (built synchronously by the first call that pairs them); per (device, stream) the
- *     int64 difference arrays of the sweep (grown on demand, SYN_ERR_OOM possible), and for
- *     calls spanning several kernel slabs a second array, a side stream and events (the
- *     finish of slab i overlaps the walk of slab i + 1; the call joins the side stream before
- *     returning); and the stream-ordered SVR scratch described at syn_model_desc.  After one
- *     call of a given shape on a stream, later such calls only enqueue work, so they may be
- *     captured into a CUDA graph.
+ *     The caller owns every buffer it passes.  The library keeps its own scratch, all of it
+ *     stream-ordered (allocated from a library-owned CUDA memory pool on the call's stream, never
+ *     with a host synchronisation): per (model, clock table) a clock-cut copy of the forest built
+ *     by k_cut_blocks on the stream of the first call that pairs them (calls on other streams wait
+ *     for its event); per (device, stream) the int64 difference arrays of the sweep, kept zeroed
+ *     between calls and grown on demand (SYN_ERR_OOM possible); for calls spanning several kernel
+ *     slabs a second array, a side stream and events (the finish of slab i overlaps the walk of
+ *     slab i + 1; the call joins the side stream before returning); and per call the general
+ *     path's and the SVR member's scratch (freed stream-ordered before the call returns).
+ *     synergy_prepare creates the persistent pieces for a shape; after it (or after one call of
+ *     that shape on a stream) later such calls only enqueue work, so they may be captured into a
+ *     CUDA graph.  A call that would have to create persistent scratch while its stream is being
+ *     captured returns SYN_ERR_UNSUPPORTED instead.
+ *   - Paths: the tree-major kernels (k_tm_walk + k_tm_finish) when every forest's leaves fit the
+ *     int64 fixed-point range and the inputs / trees fit shared memory (about F <= 90 and 25 000
+ *     trees per call); otherwise the general exact kernels (k_gen_forest + k_gen_finish: direct
+ *     traversal, 320-bit exact leaf sums), which accept every valid model and F <= 254.  Both
+ *     return the same bits.
  *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
  *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
  *   - Handles (models, clock tables, workspaces) are bound to the device they were created
@@ -48,7 +57,7 @@
 extern "C" {
 #endif
 
-#define SYNERGY_VERSION 2
+#define SYNERGY_VERSION 3
 #define SYNERGY_MAX_FREQS 4096
 #define SYNERGY_MAX_TARGETS 16
 #define SYNERGY_MAX_INPUTS 255
@@ -69,12 +78,14 @@ typedef enum {
     SYN_MIN_EDP = 2,     /* lowest E*T, T = 1/S                  (L253)             */
     SYN_MIN_ED2P = 3,    /* lowest E*T^2                         (L253)             */
     SYN_ES = 4,          /* highest speedup with E <= E_def - x%(E_def - E_min)  (L267) */
-    SYN_PL = 5           /* lowest energy with S >= S_def - x%(S_def - S(i_minE)) (L271) */
+    SYN_PL = 5,          /* lowest energy with S >= S_def - x%(S_def - S(i_minE)) (L271) */
+    SYN_ES_ABS = 6,      /* highest speedup with E <= (1 - x%) E_def; -1 if none  (L11, L46) */
+    SYN_PL_ABS = 7       /* lowest energy with S >= (1 - x%) S_def; -1 if none   (L11, L46) */
 } syn_target_kind;
 
 typedef struct {
     int32_t kind;        /* syn_target_kind                                         */
-    float x;             /* percentage in [0, 100] for SYN_ES / SYN_PL, else ignored */
+    float x;             /* percentage in [0, 100] for SYN_ES / PL / ES_ABS / PL_ABS, else ignored */
 } syn_target;
 
 typedef void *syn_stream;   /* cudaStream_t */
@@ -134,9 +145,11 @@ int32_t synergy_version(void);
 
 /* Validate, re-lay (breadth-first, children adjacent) and upload a model to `device`.
  * INVALID_ARG: null arrays, n_inputs out of range, a child id outside its tree, a node
- * reached twice (not a tree), a split feature outside [0, n_inputs), all member weights 0,
- * an SVR member with NULL arrays, n_sv outside [1, 2^24], non-finite values or a zero scale.
- * UNSUPPORTED: depth > SYNERGY_MAX_DEPTH or more than 2^31-2 nodes.  OOM / CUDA otherwise.
+ * reached twice (not a tree), a split feature outside [0, n_inputs), a non-finite leaf value,
+ * all member weights 0, an SVR member with NULL arrays, n_sv outside [1, 2^24], non-finite
+ * values or a zero scale.  (Thresholds may be any fp32, NaN included: x <= NaN is false.)
+ * UNSUPPORTED: depth > SYNERGY_MAX_DEPTH, a tree of more than 2^23 - 1 nodes or more than
+ * 2^31 - 16 nodes in all.  OOM / CUDA otherwise.
  * Synchronous (returns after the upload). */
 syn_status synergy_model_create(const syn_model_desc *desc, int32_t device, syn_model **out);
 syn_status synergy_model_destroy(syn_model *model);
@@ -150,6 +163,15 @@ syn_status synergy_clocks_create(const float *h_freqs, int32_t n_freqs, int32_t 
                                  syn_clocks **out);
 syn_status synergy_clocks_destroy(syn_clocks *clocks);
 syn_status synergy_clocks_info(const syn_clocks *clocks, int32_t *n_freqs);
+
+/* Create the persistent scratch a call of this shape needs on `stream` (clock-cut copies, the
+ * sweep's difference arrays and slab-pipeline stream), enqueueing only the k_cut_blocks builds, so
+ * that later calls with these models, this clock table, at most n_kernels kernels and this stream
+ * only enqueue kernels (e.g. inside a CUDA-graph capture).  models[0..1] speedup / energy,
+ * models[2..3] (n_models == 4) the four-model variant's direct models or NULL.  Errors as
+ * synergy_sweep4 (no feature or output buffers are needed). */
+syn_status synergy_prepare(const syn_model *const *models, int32_t n_models, int64_t n_kernels,
+                           int32_t n_features, const syn_clocks *clocks, syn_stream stream);
 
 /* Predictions for every (kernel, clock) pair:
  *   d_speedup[k][i] = (float)(mS(k, f_i) / mS(k, f_def)),  d_energy likewise with mE,
@@ -188,9 +210,7 @@ syn_status synergy_sweep(const syn_model *speedup, const syn_model *energy,
  * derived as E/S resp. E/S^2, as in synergy_sweep).  Each model is normalised by its own default-
  * clock prediction; MIN_EDP / MIN_ED2P minimise the direct model's normalised prediction (a clock
  * also needs that prediction finite and > 0).  d_pred (nullable): [4][n_kernels][n_freqs]
- * normalised predictions (rows of absent models untouched).  Runs on the exact fixed-point kernel
- * only: SYN_ERR_UNSUPPORTED when a forest's leaves exceed its int64 range (Q8).
- * Other errors as synergy_sweep. */
+ * normalised predictions (rows of absent models untouched).  Errors as synergy_sweep. */
 syn_status synergy_sweep4(const syn_model *const *models, const float *d_features, int64_t n_kernels,
                           int32_t n_features, const syn_clocks *clocks, int32_t default_idx,
                           const syn_target *h_targets, int32_t n_targets, int32_t *d_choice,
@@ -238,8 +258,9 @@ syn_status synergy_sweep_host(syn_workspace *ws, const syn_model *speedup,
                               int32_t default_idx, const syn_target *h_targets,
                               int32_t n_targets, int32_t *h_choice, syn_stream stream);
 
-/* Launch statistics of the last sweep/predict/select enqueued by this host thread (for
- * benchmarks: kernels launched, evaluations, node decisions of complete paths).  NULLs ok. */
+/* Launch statistics of the last sweep/predict/select enqueued by this host thread (for tests and
+ * benchmarks): kernels launched, evaluations, grid, block, variant (4000 = tree-major kernels,
+ * 5000 = general exact kernels, 0 = standalone kernels).  NULLs ok. */
 syn_status synergy_last_launch(int32_t *kernels_launched, int64_t *evals, int64_t *grid,
                                int32_t *block, int32_t *variant);
 
@@ -252,6 +273,14 @@ syn_status synergy_last_launch(int32_t *kernels_launched, int64_t *evals, int64_
 syn_status synergy_timing_enable(int32_t on);
 syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms, int64_t *launches,
                                int32_t *n_kernels);
+
+/* Tuning knobs (launch-configuration choices only; results are identical for every setting), for
+ * tests and benchmarks.  Initialised once from the environment (SYNERGY_<KEY upper-case>), then
+ * process-wide.  Keys: "algo" (0 automatic, 1 force the general exact kernels), "tm_kb" (k_tm_walk
+ * kernels per feature block, 32..256), "tm_ctas", "tm_nsub", "tm_dyn" (-1 automatic), "tm_pdl",
+ * "tm_slab", "tm_pipe", "tm_kt", "gen_kt", "svr_splits"; 0 = automatic unless noted.  INVALID_ARG: unknown key. */
+syn_status synergy_config_set(const char *key, int64_t value);
+syn_status synergy_config_get(const char *key, int64_t *value);
 
 #ifdef __cplusplus
 }

@@ -5,27 +5,25 @@
 
 namespace syn {
 
-// Packed forest node, 8 bytes, breadth-first per tree with the two children adjacent:
+// Packed forest node, 8 bytes, breadth-first per tree with the two children adjacent
+// (k_gen_forest's direct walks):
 //   .x = bits of the fp32 threshold (internal) or leaf value (leaf)
 //   .y = meta = (delta << 8) | code,  delta signed 24-bit
 //        code in [0, F)  : split on static feature `code`
 //        code == F       : split on the core clock (input F)
-//        code == F + 1   : leaf (the kernel's x-vector slot F+1 holds NaN, so the
-//                          comparison is false and idx += delta + 1 == idx + 0)
-//   next = idx + delta + (x <= thr ? 0 : 1);  leaves use delta = -1 (self loop).
-// With per-tree depth D every lane takes exactly D steps, branch-free, and lands on a leaf.
+//        code == F + 1   : leaf
+//   next = idx + delta + (x <= thr ? 0 : 1)
 constexpr int kCodeBits = 8;
 constexpr int kMaxDelta = (1 << 23) - 1;
 
 struct DevModel {
-    const uint2* nodes;      // [n_nodes + 1]; node n_nodes is a padding leaf (value 0)
+    const uint2* nodes;      // [n_nodes]
     const int2* trees;       // [n_trees] {first node (BFS root), depth}
     const double* lin_w;     // [n_inputs]
     double lin_b;
     double lin_weight;       // 0 => absent
     double forest_weight;    // 0 => absent
     int n_trees;
-    int pad_leaf;            // index of the padding leaf
     int depth;               // deepest root-to-leaf path over all trees (edges)
     // 2-level block layout (32 B per block, two uint4): words
     //   0: thr(n)  1: thr(c0)  2: thr(c1)  3: code(n) | code(c0) << 8 | code(c1) << 16 |
@@ -38,10 +36,13 @@ struct DevModel {
     const int* broot;        // [n_trees] root block of each tree
     int bdepth;              // max(1, ceil(depth / 2)) over all trees
     int nblk;                // blocks of all trees (tree t owns [broot[t], broot[t+1] or nblk))
-    // exact fixed-point leaf sums (k_sweep_da): every leaf v is an integer multiple of 2^-s and
-    // n_trees * max|v| * 2^s < 2^62, so v * fx_scale is an exact int64 and sums are exact
+    // exact leaf sums (Q8): every (finite) fp32 leaf v is an integer multiple of 2^-s
+    // (s from the smallest leaf ulp).  fx_ok: n_trees * max|v| * 2^s < 2^62, so v * 2^s is an
+    // exact int64 and int64 sums are exact in any order (k_tm_walk); otherwise k_gen_forest sums
+    // v * 2^s exactly in a multi-word integer accumulator.
     int fx_ok;
     int fx32;                // fx_ok and every |v| * 2^s < 2^31 (int32 fixed-point leaves fit)
+    int fx_s;                // s
     double fx_scale;         // 2^s
     double fx_inv;           // 2^-s
     // SVR_RBF member: svr = b + sum_j dual_j exp(-gamma ||(x - mean)/scale - sv_j||^2)
@@ -89,13 +90,12 @@ struct SvrArgs {
 };
 
 constexpr int kMaxTargets = 16;
-constexpr int kGrid = 1024;     // uniform bins over [f_0, f_{n-1}] for the clock-cut lookup
 
 enum Mode : int { kModePredict = 0, kModeSweep = 1 };
 
 struct SweepArgs {
     DevModel ms, me;         // speedup, energy
-    DevModel mx[2];          // four-model variant: direct EDP, ED2P models (k_sweep_da only)
+    DevModel mx[2];          // four-model variant: direct EDP, ED2P models
     int has_x[2];            // which of mx are present
     const float* features;   // [n_k][F]
     long long n_k;
@@ -111,22 +111,8 @@ struct SweepArgs {
     float* E_out;
     float* X_out[2];         // direct EDP / ED2P normalised predictions, [n_k][n_f] or null
     int mode;
-    int tile_k;              // kernels per CTA
+    int tile_k;              // kernels per finish CTA
     int xs;                  // x-vector stride in smem (floats)
-    // clock-interval traversal (k_sweep_iv) only
-    int tc;                  // trees per chunk (one (kernel, tree) task per thread)
-    int words;               // ceil(n_f / 32) run-start mask words per task
-    int vcap;                // run values kept per task
-    int vs;                  // run-value stride per task (odd, conflict-free)
-    int region;              // bytes of the task region (also holds the float finish scratch)
-    // warp-streaming (k_sweep_ws) only
-    int win;                 // ring-window slots per warp
-    int slot_bytes;          // bytes per slot
-    int head_bytes;          // bytes of the staged clocks / features / grid head
-    // clock-cut grid built once per clock table (syn_clocks)
-    const unsigned short* grid;   // [kGrid + 1]
-    float f0, inv_step;
-    int nsub;                // k_sweep_da: clock sub-ranges per (kernel, tree) task (small batches)
 };
 
 struct SelectArgs {

@@ -1,100 +1,27 @@
-// kernels.cuh — sm_100a kernels of the SYnergy predict+select hot path.
+// kernels.cuh — shared finish / selection kernels of the SYnergy predict+select hot path (sm_100a).
 //
-//   k_sweep<SLOTS, TILP>  fused: model inference for every (kernel, clock) pair of a CTA's
-//                         kernel tile, default-clock normalisation (L69), then
-//                         per-target objective + masked lowest-index argmin (L253-L271, L322)
-//                         with warp shuffles; predictions stay in shared memory unless asked.
-//   k_select              standalone selection over predictions in HBM (one warp per kernel).
+//   combine()        a model's raw output from its exact forest sum: linear member, forest mean
+//                    (Q7/Q8)
+//   finish_tile4()   SVR member, default-clock normalisation (L69), then per target the objective /
+//                    constraint and the masked lowest-index argmin (L253-L271, L322) with warp
+//                    shuffles; used by k_tm_finish and k_gen_finish
+//   k_select         standalone selection over predictions in HBM (one warp per kernel)
+//   k_pareto, k_choice_error, k_error_reduce, k_plan   NEXT f3 / f4 (Pareto front, choice error,
+//                    plan emission)
 //
-// Arithmetic contract (Q15): identical op sequence to the oracle — fp64 fma chain
-// for the linear member, fp64 sum of fp32 leaves in tree order, fp64 division by T, fp64
-// normalisation rounded once to fp32, fp64 keys/thresholds; every fp64 op is an explicit
-// _rn intrinsic so nothing is contracted.  Ties: lexicographic (key, index) minimum.
+// Arithmetic contract (Q15): the oracle's op sequence — fp64 fma chain for the linear
+// member, exact leaf sum rounded once then / T, fp64 normalisation rounded once to fp32, fp64
+// keys / thresholds; every fp64 op is an explicit _rn intrinsic and the library is built with
+// --fmad=false, so nothing is contracted.  Ties: lexicographic (key, index) minimum.
 #pragma once
-#include <cuda_runtime.h>
-#include <math_constants.h>
-#include <cstdint>
-
-#include "internal.h"
+#include "device_util.cuh"
 #include "kernels_svr.cuh"
 
 namespace syn {
 
-__device__ __forceinline__ uint2 ldg_node(const uint2* p) {
-    uint2 r;
-    asm volatile("ld.global.nc.v2.u32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
-    return r;
-}
-
 __device__ __forceinline__ bool valid_pred(float s, float e) {
     // DESIGN.md Q16: finite and strictly positive speedup and energy
     return isfinite(s) && isfinite(e) && s > 0.0f && e > 0.0f;
-}
-
-// Raw model output for SLOTS (kernel, clock) units held by this thread.
-//   xk[row[s] + j] = static feature j of the unit's kernel, slot F+1 = NaN (leaf code)
-template <int SLOTS, int TILP>
-__device__ __forceinline__ void eval_model(const DevModel& m, const float* __restrict__ xk,
-                                           const int (&row)[SLOTS], const float (&f)[SLOTS],
-                                           int F, double (&out)[SLOTS]) {
-#pragma unroll
-    for (int s = 0; s < SLOTS; ++s) out[s] = 0.0;
-    if (m.lin_weight != 0.0) {
-        // Linear / Lasso member (L386): lin = b; lin = fma(w_j, x_j, lin), j = 0..F in order
-#pragma unroll
-        for (int s = 0; s < SLOTS; ++s) {
-            double lin = m.lin_b;
-            for (int j = 0; j < F; ++j) lin = __fma_rn(__ldg(m.lin_w + j), (double)xk[row[s] + j], lin);
-            lin = __fma_rn(__ldg(m.lin_w + F), (double)f[s], lin);
-            out[s] = __dadd_rn(out[s], m.lin_weight == 1.0 ? lin : __dmul_rn(m.lin_weight, lin));
-        }
-    }
-    if (m.forest_weight != 0.0) {
-        // Random Forest member (L386): mean of T trees, x <= thr goes left (Q8, Q9)
-        double acc[SLOTS];
-#pragma unroll
-        for (int s = 0; s < SLOTS; ++s) acc[s] = 0.0;
-        for (int t0 = 0; t0 < m.n_trees; t0 += TILP) {
-            const int nt = min(TILP, m.n_trees - t0);
-            int idx[TILP][SLOTS];
-            int depth = 0;
-#pragma unroll
-            for (int j = 0; j < TILP; ++j) {
-                int2 td = (j < nt) ? __ldg(m.trees + t0 + j) : make_int2(m.pad_leaf, 0);
-                depth = max(depth, td.y);
-#pragma unroll
-                for (int s = 0; s < SLOTS; ++s) idx[j][s] = td.x;
-            }
-            // depth is uniform across the CTA: every lane takes the same number of steps,
-            // lanes that reached a leaf early self-loop on it (no divergence)
-            for (int d = 0; d < depth; ++d) {
-#pragma unroll
-                for (int j = 0; j < TILP; ++j) {
-#pragma unroll
-                    for (int s = 0; s < SLOTS; ++s) {
-                        const uint2 n = ldg_node(m.nodes + idx[j][s]);
-                        const int code = (int)(n.y & 0xffu);
-                        const float xs = xk[row[s] + code];
-                        const float x = (code == F) ? f[s] : xs;
-                        idx[j][s] += ((int)n.y >> kCodeBits) + (x <= __uint_as_float(n.x) ? 0 : 1);
-                    }
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < TILP; ++j) {
-                if (j < nt) {   // uniform guard; accumulation strictly in tree order
-#pragma unroll
-                    for (int s = 0; s < SLOTS; ++s)
-                        acc[s] = __dadd_rn(acc[s], (double)__uint_as_float(ldg_node(m.nodes + idx[j][s]).x));
-                }
-            }
-        }
-#pragma unroll
-        for (int s = 0; s < SLOTS; ++s) {
-            const double forest = __ddiv_rn(acc[s], (double)m.n_trees);
-            out[s] = __dadd_rn(out[s], m.forest_weight == 1.0 ? forest : __dmul_rn(m.forest_weight, forest));
-        }
-    }
 }
 
 __device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
@@ -104,6 +31,23 @@ __device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
         const int oi = __shfl_xor_sync(0xffffffffu, idx, off);
         if (ok < key || (ok == key && oi < idx)) { key = ok; idx = oi; }
     }
+}
+
+// Model output from its forest sum (the exact leaf sum rounded once to fp64; oracle order: linear
+// member first, then the forest mean; a weight of exactly 1 skips its multiplication, Q7).
+__device__ __forceinline__ double combine(const DevModel& m, double forest_sum, const float* xrow, float f, int F) {
+    double out = 0.0;
+    if (m.lin_weight != 0.0) {
+        double lin = m.lin_b;
+        for (int j = 0; j < F; ++j) lin = __fma_rn(__ldg(m.lin_w + j), (double)xrow[j], lin);
+        lin = __fma_rn(__ldg(m.lin_w + F), (double)f, lin);
+        out = __dadd_rn(out, m.lin_weight == 1.0 ? lin : __dmul_rn(m.lin_weight, lin));
+    }
+    if (m.forest_weight != 0.0) {
+        const double forest = __ddiv_rn(forest_sum, (double)m.n_trees);
+        out = __dadd_rn(out, m.forest_weight == 1.0 ? forest : __dmul_rn(m.forest_weight, forest));
+    }
+    return out;
 }
 
 // Selection baselines of one row (Q14-Q16): returns false if the default clock's
@@ -135,6 +79,9 @@ __device__ __forceinline__ int select_target(const float* S, const float* E, con
     const double frac = __ddiv_rn((double)x, 100.0);
     const double thr_es = __dsub_rn(E_def, __dmul_rn(frac, __dsub_rn(E_def, E_min)));
     const double thr_pl = __dsub_rn(S_def, __dmul_rn(frac, __dsub_rn(S_def, S_minE)));
+    // absolute-saving reading (L11/L46, Q1): E <= (1 - x%) E_def, S >= (1 - x%) S_def
+    const double thr_es_abs = __dmul_rn(__dsub_rn(1.0, frac), E_def);
+    const double thr_pl_abs = __dmul_rn(__dsub_rn(1.0, frac), S_def);
     double bk = CUDART_INF;
     int bx = INT_MAX;
     for (int i = lane; i < n_f; i += 32) {
@@ -155,7 +102,9 @@ __device__ __forceinline__ int select_target(const float* S, const float* E, con
                 else key = __ddiv_rn(__ddiv_rn(e, s), s);
                 break;
             case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
-            default: feas = (s >= thr_pl); key = e; break;             // PL_x
+            case 5: feas = (s >= thr_pl); key = e; break;              // PL_x
+            case 6: feas = (e <= thr_es_abs); key = -s; break;         // ES_ABS_x
+            default: feas = (s >= thr_pl_abs); key = e; break;         // PL_ABS_x
         }
         if (feas && (key < bk || (key == bk && i < bx))) { bk = key; bx = i; }
     }
@@ -244,70 +193,6 @@ __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* 
     }
 }
 
-// Two-model finish (speedup, energy).
-__device__ __forceinline__ void finish_tile(const SweepArgs& a, double* mS, double* mE,
-                                            float* sS, float* sE, int nk, long long k0) {
-    double* mv[4] = {mS, mE, nullptr, nullptr};
-    float* sv[4] = {sS, sE, nullptr, nullptr};
-    finish_tile4(a, mv, sv, nk, k0);
-}
-
-template <int SLOTS, int TILP>
-__global__ void __launch_bounds__(512) k_sweep(const __grid_constant__ SweepArgs a) {
-    extern __shared__ __align__(16) unsigned char smem[];
-    const int tile = a.tile_k;
-    const long long k0 = (long long)blockIdx.x * tile;
-    const int nk = (int)min((long long)tile, a.n_k - k0);
-    const int n_f = a.n_f;
-    const int F = a.F;
-    const int XS = a.xs;
-    double* mS = reinterpret_cast<double*>(smem);
-    double* mE = mS + (size_t)tile * n_f;
-    float* sS = reinterpret_cast<float*>(mE + (size_t)tile * n_f);
-    float* sE = sS + (size_t)tile * n_f;
-    float* xk = sE + (size_t)tile * n_f;
-    float* fr = xk + (size_t)tile * XS;
-
-    // stage the tile's feature rows (coalesced) and the clock table
-    const float* gfeat = a.features + k0 * F;
-    for (int e = threadIdx.x; e < nk * F; e += blockDim.x) {
-        const int r = e / F;
-        xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
-    }
-    for (int r = threadIdx.x; r < nk; r += blockDim.x) {
-        xk[r * XS + F] = 0.0f;
-        xk[r * XS + F + 1] = CUDART_NAN_F;     // leaf code slot
-    }
-    for (int i = threadIdx.x; i < n_f; i += blockDim.x) fr[i] = __ldg(a.freqs + i);
-    __syncthreads();
-
-    // phase 1: every (kernel, clock) unit of the tile -> raw fp64 model outputs
-    const int units = nk * n_f;
-    for (int u0 = 0; u0 < units; u0 += blockDim.x * SLOTS) {
-        int row[SLOTS];
-        float f[SLOTS];
-#pragma unroll
-        for (int s = 0; s < SLOTS; ++s) {
-            const int u = u0 + threadIdx.x + s * blockDim.x;
-            const int uu = u < units ? u : 0;
-            const int kl = uu / n_f;
-            row[s] = kl * XS;
-            f[s] = fr[uu - kl * n_f];
-        }
-        double vS[SLOTS], vE[SLOTS];
-        eval_model<SLOTS, TILP>(a.ms, xk, row, f, F, vS);
-        eval_model<SLOTS, TILP>(a.me, xk, row, f, F, vE);
-#pragma unroll
-        for (int s = 0; s < SLOTS; ++s) {
-            const int u = u0 + threadIdx.x + s * blockDim.x;
-            if (u < units) { mS[u] = vS[s]; mE[u] = vE[s]; }
-        }
-    }
-    __syncthreads();
-
-    finish_tile(a, mS, mE, sS, sE, nk, k0);
-}
-
 // Standalone selection: one warp per kernel row, rows read from HBM (L1-resident across the
 // per-target passes).  Grid-stride over kernels.
 __global__ void __launch_bounds__(256) k_select(const __grid_constant__ SelectArgs a) {
@@ -344,8 +229,8 @@ __global__ void __launch_bounds__(256) k_pareto(const float* __restrict__ S, con
 __device__ __forceinline__ double target_objective(int kind, float s, float e) {
     const double ds = (double)s, de = (double)e;
     switch (kind) {
-        case 0: case 4: return ds;
-        case 1: case 5: return de;
+        case 0: case 4: case 6: return ds;
+        case 1: case 5: case 7: return de;
         case 2: return __ddiv_rn(de, ds);
         default: return __ddiv_rn(__ddiv_rn(de, ds), ds);
     }

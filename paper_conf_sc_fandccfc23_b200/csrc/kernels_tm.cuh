@@ -1,17 +1,18 @@
 // kernels_tm.cuh — tree-major resume-walk sweep (k_tm_walk + k_tm_finish), the default fused path.
 //
-// What is computed is k_sweep_da's (kernels_da.cuh): per (kernel, model) the exact fixed-point sum
-// over trees of the leaf each clock reaches (Q8), accumulated as a difference array over
-// the clock axis, then the forest mean, linear / SVR members, default-clock normalisation and the
-// per-target masked argmin.  What changes is how the work is laid
-// on the machine, to cut L1 wavefronts, the resource k_sweep_da saturates (profiles/r1):
+// Computes, per (kernel, model), the exact fixed-point sum over trees of the leaf each clock
+// reaches (Q8), accumulated as a difference array over the clock axis, then the forest
+// mean, linear / SVR members, default-clock normalisation and the per-target masked argmin (PAPER
+// L253-L271, L316-L322).  Needs every forest within the int64 fixed-point range (fx_ok) and the
+// shared-memory limits checked by the host (tm_eligible); kernels_gen.cuh takes the rest.  The
+// work is laid on the machine to cut L1 wavefronts, the resource a kernel-major walk saturates:
 //
 //  * Tree-major lanes.  A lane task is one (kernel, model, tree).  Tasks are numbered
 //      j = ((kernel block) * TT + tree) * KB + kernel-in-block
 //    and every CTA owns a contiguous range of j, so the lanes of an SM walk the SAME few trees for
 //    up to KB different kernels at once: the SM's L1 holds those trees, the 32 lanes of a warp
 //    load blocks of one tree (shared lines), and lines are reused by every kernel of the block.
-//    (k_sweep_da instead runs ~1000 different trees per SM and hits L1 9% of the time on c3.)
+//    (round 1's kernel-major k_sweep_da ran ~1000 different trees per SM: 9% L1 hits on c3.)
 //
 //  * Resume walks.  For a fixed kernel a tree is a step function of the clock index.  walk(lo)
 //    follows clock lo's path; the run is [lo, hi) with hi = #{i : f_i <= thr} minimised over the
@@ -46,7 +47,7 @@
 //    clock), rounds it once, combines the members and runs finish_tile4; it zeroes D as it reads
 //    it, so the next call starts from zeros without a memset.
 #pragma once
-#include "kernels_da.cuh"
+#include "kernels.cuh"
 
 namespace syn {
 
@@ -118,20 +119,21 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     constexpr unsigned kEnt = 4u * NT;                                       // bytes between stack entries
     float* const xcol = xs + threadIdx.x;
     const unsigned xclk_a = su32(xcol + (size_t)F * NT);
+    xcol[(size_t)(F + 1) * NT] = 0.0f;   // folded-leaf row: either outcome reaches the same leaf
 
-    const int T0 = da_trees(a, 0), T1 = da_trees(a, 1), T2 = t.nm > 2 ? da_trees(a, 2) : 0,
-              T3 = t.nm > 2 ? da_trees(a, 3) : 0;
+    const int T0 = trees_of(a, 0), T1 = trees_of(a, 1), T2 = t.nm > 2 ? trees_of(a, 2) : 0,
+              T3 = t.nm > 2 ? trees_of(a, 3) : 0;
     const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
     const int NS = t.nsub;
     const long long per_kb = (long long)TT * NS * KB;
     for (int q = threadIdx.x; q < TT; q += NT) {
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
-        stree[q] = make_int2(__ldg(da_model(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3))), mi);
+        stree[q] = make_int2(__ldg(model_of(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3))), mi);
     }
     if (threadIdx.x < 4) {
         const int m = threadIdx.x;
         if (m < 2 || t.nm > 2) {
-            const DevModel& d = da_model(a, m);
+            const DevModel& d = model_of(a, m);
             s_blocks[m] = d.blocks;
             s_slot[m] = t.slot_of[m] * n_f;
             s_fx[m] = d.fx32;
@@ -348,7 +350,7 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
     for (int p = warp; p < NM * nk; p += nw) {                                // p = kernel * NM + model
         const int pk = p / NM, pm = p - pk * NM;
         if (pm >= 2 && !a.has_x[pm - 2]) continue;
-        const DevModel& m = da_model(a, pm);
+        const DevModel& m = model_of(a, pm);
         double* out = mv0 + ((size_t)pm * KT + pk) * n_f;
         const float* xrow = xk + pk * XS;
         const int slot = t.slot_of[pm];

@@ -1,5 +1,7 @@
 // synergy.cu — C-ABI implementation (include/synergy.h): validation, model packing, launch
-// configuration and the host-buffer end-to-end path.  All compute runs in kernels.cuh.
+// configuration, library-owned scratch and the host-buffer end-to-end path.  All compute runs in
+// the kernels: kernels_tm.cuh (default tree-major path), kernels_gen.cuh (general exact path),
+// kernels_svr.cuh (SVR member), kernels.cuh (finish, selection, Pareto, choice error, plan).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -17,15 +19,23 @@
 
 #include "internal.h"
 #include "kernels.cuh"
-#include "kernels_iv.cuh"
-#include "kernels_ws.cuh"
-#include "kernels_da.cuh"
+#include "kernels_gen.cuh"
 #include "kernels_svr.cuh"
 #include "kernels_tm.cuh"
-#include "kernels_tr.cuh"
 #include "synergy.h"
 
 using namespace syn;
+
+namespace {
+constexpr int kMaxDevices = 64;
+}
+
+struct CutCopy {                 // clock-cut copy of a model's blocks for one clock table
+    long long uid;               // syn_clocks uid
+    uint4* p;
+    cudaStream_t built_on;       // stream the k_cut_blocks build was enqueued on
+    cudaEvent_t ready;           // recorded after the build; null once known complete
+};
 
 struct syn_model {
     int device;
@@ -37,18 +47,14 @@ struct syn_model {
     void* alloc;
     DevModel dm;
     long long n_blocks;                                   // 2-level blocks (2 x uint4 each)
-    std::vector<std::pair<long long, uint4*>> cut_blocks;  // per clock table (uid): k_cut_blocks copy
-    std::vector<std::pair<long long, uint4*>> tr_blocks;   // per clock table (uid): k_tr_layout copy
-    long long max_tree_blocks;                            // blocks of the largest tree
+    std::vector<CutCopy> cuts;                            // per clock table
 };
 
 struct syn_clocks {
     int device;
     int n_f;
     float* d_freqs;
-    unsigned short* d_grid;   // clock-cut hint table, kGrid + 1 entries
-    float f0, inv_step;
-    long long uid;            // unique per created table (keys the models' clock-cut block copies)
+    long long uid;            // unique per created table (keys the models' clock-cut copies)
 };
 
 struct syn_workspace {
@@ -70,6 +76,10 @@ struct LaunchInfo {
     int variant;
 };
 thread_local LaunchInfo g_last = {0, 0, 0, 0, 0};
+
+// Variant codes reported by synergy_last_launch (tests / bench read which path ran).
+constexpr int kVarTm = 4000;      // k_tm_walk + k_tm_finish
+constexpr int kVarGen = 5000;     // k_gen_forest + k_gen_finish
 
 // Optional per-kernel device timing (synergy_timing_enable): CUDA events recorded on the launch
 // stream around every library kernel launch; read back (summed per kernel) by synergy_timing_read.
@@ -155,242 +165,152 @@ bool current_device_is(int dev) {
     return cudaGetDevice(&cur) == cudaSuccess && cur == dev;
 }
 
-int sm_count(int dev) {
-    static int cached[64] = {0};
-    if (dev < 0 || dev >= 64) return 148;
-    if (!cached[dev]) {
+// ------------------------------------------------------------------------ tuning knobs
+// Read once from the environment (SYNERGY_<NAME>) at first use; synergy_config_set changes them
+// at run time (tests use it to force launch-configuration variants).  0 / -1 = automatic.
+struct Knobs {
+    std::atomic<long long> algo{0};       // 0 auto, 1 force k_gen (general exact path)
+    std::atomic<long long> tm_kb{0};      // k_tm_walk kernels per feature block (32..256)
+    std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default 2 per SM)
+    std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
+    std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
+    std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
+    std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
+    std::atomic<long long> tm_pipe{1};    // slab pipeline (finish on a side stream)
+    std::atomic<long long> tm_kt{0};      // k_tm_finish kernels per CTA
+    std::atomic<long long> gen_kt{0};     // k_gen_finish kernels per CTA
+    std::atomic<long long> svr_splits{0}; // k_svr SV-range splits (0: fill the SMs)
+};
+Knobs g_knobs;
+struct KnobName {
+    const char* name;
+    std::atomic<long long>* v;
+};
+const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
+                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
+                           {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
+                           {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits}};
+std::once_flag g_knobs_once;
+
+const Knobs& knobs() {
+    std::call_once(g_knobs_once, [] {
+        for (const KnobName& k : kKnobs) {
+            char env[64] = "SYNERGY_";
+            for (int i = 0; k.name[i] && i < 40; ++i) env[8 + i] = (char)toupper(k.name[i]), env[9 + i] = 0;
+            const char* v = getenv(env);
+            if (v && *v) k.v->store(atoll(v));
+        }
+    });
+    return g_knobs;
+}
+
+// -------------------------------------------------------------------- per-device state
+struct DevState {
+    std::once_flag once;
+    int sms = 148;
+    int optin = 227 * 1024;               // max dynamic shared memory per CTA (opt-in)
+    cudaError_t init_err = cudaSuccess;
+    cudaMemPool_t pool = nullptr;         // library-owned stream-ordered pool (release threshold max)
+    std::mutex occ_mu;
+    std::vector<std::pair<size_t, int>> finish_occ;   // k_tm_finish: (smem bytes, CTAs per SM)
+};
+DevState g_dev[kMaxDevices];
+
+template <typename K>
+cudaError_t allow_smem(K kernel, int bytes) {
+    return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+}
+
+// Once per device (the attribute is per device): query limits, opt every kernel with dynamic
+// shared memory in to the device maximum, create the library pool.
+DevState* dev_state(int dev) {
+    if (dev < 0 || dev >= kMaxDevices) return nullptr;
+    DevState& d = g_dev[dev];
+    std::call_once(d.once, [&d, dev] {
+        DeviceGuard g(dev);
         int v = 0;
-        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0) v = 148;
-        cached[dev] = v;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0) d.sms = v;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) == cudaSuccess && v > 0) d.optin = v;
+        cudaError_t e = cudaSuccess;
+        auto chk = [&e](cudaError_t x) { if (e == cudaSuccess) e = x; };
+        chk(allow_smem(k_tm_walk<kTmNT, true>, d.optin));
+        chk(allow_smem(k_tm_walk<kTmNT, false>, d.optin));
+        chk(allow_smem(k_tm_finish, d.optin));
+        chk(allow_smem(k_svr<1>, d.optin));
+        chk(allow_smem(k_svr<2>, d.optin));
+        chk(allow_smem(k_svr<3>, d.optin));
+        chk(allow_smem(k_svr<4>, d.optin));
+        chk(allow_smem(k_svr<5>, d.optin));
+        chk(allow_smem(k_svr<6>, d.optin));
+        chk(allow_smem(k_svr<7>, d.optin));
+        chk(allow_smem(k_svr<8>, d.optin));
+        chk(allow_smem(k_svr_u, d.optin));
+        cudaMemPoolProps props;
+        memset(&props, 0, sizeof props);
+        props.allocType = cudaMemAllocationTypePinned;
+        props.handleTypes = cudaMemHandleTypeNone;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        if (e == cudaSuccess) {
+            chk(cudaMemPoolCreate(&d.pool, &props));
+            if (e == cudaSuccess) {
+                unsigned long long thr = ~0ULL;
+                chk(cudaMemPoolSetAttribute(d.pool, cudaMemPoolAttrReleaseThreshold, &thr));
+            }
+        }
+        if (e != cudaSuccess) cudaGetLastError();
+        d.init_err = e;
+    });
+    return &d;
+}
+
+syn_status need_dev(int dev, DevState** out) {
+    DevState* d = dev_state(dev);
+    if (!d) return fail(SYN_ERR_INVALID_ARG, "device %d out of range", dev);
+    if (d->init_err != cudaSuccess) return cuda_fail(d->init_err, "device setup");
+    *out = d;
+    return SYN_OK;
+}
+
+bool capturing(cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cs) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
     }
-    return cached[dev];
+    return cs != cudaStreamCaptureStatusNone;
+}
+
+syn_status pool_alloc(DevState* d, size_t bytes, cudaStream_t st, void** out, const char* what) {
+    cudaError_t e = cudaMallocFromPoolAsync(out, std::max<size_t>(bytes, 256), d->pool, st);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *out = nullptr;
+        return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "%s: %zu bytes", what, bytes) : cuda_fail(e, what);
+    }
+    return SYN_OK;
 }
 
 syn_status check_targets(const syn_target* t, int32_t n_t) {
     if (n_t < 1 || n_t > SYNERGY_MAX_TARGETS) return fail(SYN_ERR_INVALID_ARG, "n_targets=%d outside [1, %d]", n_t, SYNERGY_MAX_TARGETS);
     if (!t) return fail(SYN_ERR_INVALID_ARG, "h_targets is NULL");
     for (int i = 0; i < n_t; ++i) {
-        if (t[i].kind < SYN_MAX_PERF || t[i].kind > SYN_PL) return fail(SYN_ERR_INVALID_ARG, "target %d: unknown kind %d", i, t[i].kind);
-        if ((t[i].kind == SYN_ES || t[i].kind == SYN_PL) && !(t[i].x >= 0.0f && t[i].x <= 100.0f))
+        if (t[i].kind < SYN_MAX_PERF || t[i].kind > SYN_PL_ABS) return fail(SYN_ERR_INVALID_ARG, "target %d: unknown kind %d", i, t[i].kind);
+        if (t[i].kind >= SYN_ES && !(t[i].x >= 0.0f && t[i].x <= 100.0f))
             return fail(SYN_ERR_INVALID_ARG, "target %d: x=%g outside [0, 100]", i, (double)t[i].x);
     }
     return SYN_OK;
 }
 
-// ---------------------------------------------------------------- launch configuration
-
-struct Config {
-    int algo;                 // 0 = direct traversal (k_sweep), 1 = clock-interval (k_sweep_iv)
-    int slots, tilp, tile_k, nt, xs;
-    int tc, words, vcap, vs, region;
-    int win, slot_bytes, head_bytes;
-    size_t smem;
-};
-
-int env_int(const char* name, int dflt) {
-    const char* v = getenv(name);
-    return (v && *v) ? atoi(v) : dflt;
-}
-
-size_t sweep_smem(int tile_k, int n_f, int xs) {
-    return (size_t)tile_k * ((size_t)n_f * 24 + (size_t)xs * 4) + (size_t)n_f * 4;
-}
-
-// Choose per-thread slots (units in flight) and trees-in-flight so that the grid keeps every
-// SM busy for small batches (slots=1, 4 trees in flight) and amortises staging for large ones.
-Config choose_config(long long n_k, int n_f, int F, int dev) {
-    Config c;
-    c.algo = 0;
-    c.tc = c.words = c.vcap = c.vs = c.region = 0;
-    c.win = c.slot_bytes = c.head_bytes = 0;
-    const long long resident = (long long)sm_count(dev) * 2048;
-    const long long evals = n_k * (long long)n_f;
-    c.slots = evals >= 16 * resident ? 8 : evals >= 8 * resident ? 4 : evals >= 4 * resident ? 2 : 1;
-    c.tilp = c.slots <= 2 ? 4 : c.slots == 4 ? 2 : 1;
-    c.xs = (F + 2) | 1;   // odd stride: rows of different kernels land in different banks
-    long long tk = std::max(1, (256 * c.slots) / n_f);
-    tk = std::min<long long>(tk, std::max<long long>(n_k, 1));
-    while (tk > 1 && sweep_smem((int)tk, n_f, c.xs) > 200 * 1024) --tk;
-    c.tile_k = (int)tk;
-    long long thr = (c.tile_k * (long long)n_f + c.slots - 1) / c.slots;
-    thr = (thr + 31) / 32 * 32;
-    c.nt = (int)std::min<long long>(std::max<long long>(thr, 32), 512);
-    c.smem = sweep_smem(c.tile_k, n_f, c.xs);
-    return c;
-}
-
-// Clock-interval kernel: NT threads, TK kernels per CTA, TC = NT / TK trees per chunk (one
-// (kernel, tree) task per thread), accumulators for the TK x n_f units in shared memory.
-// Small batches use TK = 1 so the grid spans the SMs; large ones TK = 4 so a chunk's trees are
-// shared by more kernels (L1 reuse of the upper levels).
-size_t iv_smem(int nt, int tk, int n_f, int xs, int words, int vs, int* region) {
-    const int tc = std::max(1, nt / tk);
-    size_t tasks = (size_t)tc * tk * ((size_t)words * 8 + (size_t)vs * 8);
-    tasks = std::max(tasks, (size_t)tk * n_f * 8);            // finish-phase float scratch
-    tasks = (tasks + 15) & ~(size_t)15;
-    *region = (int)tasks;
-    return (size_t)tk * n_f * 16 + tasks + (size_t)n_f * 4 + (size_t)tk * xs * 4 + (kGrid + 1) * 2 + 16;
-}
-
-bool choose_iv(long long n_k, int n_f, int F, int dev, Config& c) {
-    if (n_f > 1024) return false;
-    const int sms = sm_count(dev);
-    c.nt = env_int("SYNERGY_NT", 128) >= 256 ? 256 : 128;
-    int tk = (int)std::min<long long>(4, std::max<long long>(1, n_k / (8LL * sms)));
-    tk = env_int("SYNERGY_TK", tk);
-    tk = (int)std::max<long long>(1, std::min<long long>(std::min(tk, c.nt), std::max<long long>(n_k, 1)));
-    c.algo = 1;
-    c.slots = 0;
-    c.tilp = 0;
-    c.tile_k = tk;
-    c.xs = (F + 2) | 1;
-    c.tc = std::max(1, c.nt / tk);
-    c.words = (n_f + 31) / 32;
-    c.vcap = std::max(1, env_int("SYNERGY_VCAP", 24));
-    c.vs = c.vcap | 1;
-    c.smem = iv_smem(c.nt, tk, n_f, c.xs, c.words, c.vs, &c.region);
-    return c.smem <= 220 * 1024;
-}
-
-template <int NT, int MINB>
-cudaError_t launch_iv_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    static size_t smem_set = 48 * 1024;
-    if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep_iv<NT, MINB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
-        if (e != cudaSuccess) return e;
-        smem_set = c.smem;
-    }
-    k_sweep_iv<NT, MINB><<<(unsigned)grid, NT, c.smem, st>>>(a);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_iv(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    return c.nt == 256 ? launch_iv_t<256, 4>(a, c, grid, st) : launch_iv_t<128, 8>(a, c, grid, st);
-}
-
-// Warp-streaming kernel: KPC kernels per CTA, one warp per (kernel, model), WIN-slot ring
-// window of finished trees per warp, accumulators in registers (n_f <= 256).
-bool choose_ws(long long n_k, int n_f, int F, int dev, Config& c) {
-    if (n_f > 256) return false;
-    int kpc = env_int("SYNERGY_KPC", 2);
-    kpc = std::max(1, std::min(kpc, 4));
-    kpc = (int)std::min<long long>(kpc, std::max<long long>(n_k, 1));
-    c.algo = 2;
-    c.slots = 0;
-    c.tilp = 0;
-    c.tile_k = kpc;
-    c.nt = 64 * kpc;
-    c.xs = (F + 2) | 1;
-    c.words = (n_f + 31) / 32;
-    c.vcap = std::max(1, env_int("SYNERGY_VCAP", 32));
-    c.vs = c.vcap;
-    int win = std::max(32, std::min(1024, env_int("SYNERGY_WIN", 64)));
-    c.win = 32;
-    while (c.win * 2 <= win) c.win *= 2;                 // power of two: slot = tree & (WIN-1)
-    int sb = c.vs * 4 + c.words * 4 + 8;
-    c.slot_bytes = (sb + 7) & ~7;
-    c.head_bytes = (int)((((size_t)(n_f + kpc * c.xs) * 4 + (kGrid + 1) * 2) + 15) & ~(size_t)15);
-    const size_t slots = (size_t)2 * kpc * c.win * c.slot_bytes;
-    const size_t fin = (size_t)kpc * n_f * 24;
-    c.smem = c.head_bytes + std::max(slots, fin);
-    c.tc = c.region = 0;
-    return c.smem <= 220 * 1024;
-}
-
-template <int CL>
-cudaError_t launch_ws_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    static size_t smem_set = 48 * 1024;
-    if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep_ws<CL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
-        if (e != cudaSuccess) return e;
-        smem_set = c.smem;
-    }
-    k_sweep_ws<CL><<<(unsigned)grid, c.nt, c.smem, st>>>(a);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_ws(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    if (c.words <= 2) return launch_ws_t<2>(a, c, grid, st);
-    if (c.words <= 4) return launch_ws_t<4>(a, c, grid, st);
-    return launch_ws_t<8>(a, c, grid, st);
-}
-
-// Difference-array kernel: KPC kernels per CTA, exact int64 leaf sums (needs fx_ok forests).
-// KPC grows when a kernel has fewer trees than the CTA has threads, so lanes keep walking and
-// the per-CTA staging / finish is amortised.
-size_t da_head(int nt, int kpc, int n_f, int xs, int nm) {
-    const size_t h = (size_t)kpc * nm * (n_f + 1) * 8 + (size_t)nt * kpc * nm * 8 + (size_t)nm * kpc * n_f * 12 +
-                     (size_t)n_f * 4 + (size_t)kpc * xs * 4 + (size_t)(kGrid + 2) * 2 + 16;
-    return (h + 15) & ~(size_t)15;
-}
-
-// The per-thread top-block cache (TOPC) is only allocated when enabled: shared memory comes out of
-// the same 256 KB as L1, and this kernel lives on L1 hits of the upper tree blocks.
-bool da_topc() { return env_int("SYNERGY_TOPC", 0) != 0; }
-
-size_t da_smem(int nt, int kpc, int n_f, int xs, int nm) {
-    return da_head(nt, kpc, n_f, xs, nm) + (da_topc() ? (size_t)nt * 160 : 0);
-}
-
-bool choose_da(const syn_model* sp, const syn_model* en, long long n_k, int n_f, int F, Config& c,
-               const syn_model* x2 = nullptr, const syn_model* x3 = nullptr) {
-    if (n_f > 2048) return false;
-    if ((sp->n_trees && !sp->dm.fx_ok) || (en->n_trees && !en->dm.fx_ok)) return false;
-    if ((x2 && x2->n_trees && !x2->dm.fx_ok) || (x3 && x3->n_trees && !x3->dm.fx_ok)) return false;
-    const int nm = (x2 || x3) ? 4 : 2;
-    const int tt = std::max(1, sp->n_trees + en->n_trees + (x2 ? x2->n_trees : 0) + (x3 ? x3->n_trees : 0));
-    int nt = env_int("SYNERGY_NT", 128);
-    nt = nt >= 256 ? 256 : (nt >= 128 ? 128 : 64);
-    int kpc = tt >= nt ? 1 : (3 * nt + 2 * tt - 1) / (2 * tt);      // ~1.5 tasks per thread
-    kpc = (int)std::min<long long>(kpc, std::max<long long>(1, n_k / (2LL * sm_count(0))));   // fill the SMs
-    kpc = env_int("SYNERGY_KPC", kpc);
-    kpc = (int)std::max<long long>(1, std::min<long long>(std::min(kpc, 16), std::max<long long>(n_k, 1)));
-    c.algo = 3;
-    c.tilp = 0;
-    c.tile_k = kpc;
-    c.nt = nt;
-    c.xs = (F + 2) | 1;
-    c.tc = c.words = c.vcap = c.vs = c.region = 0;
-    c.win = c.slot_bytes = c.head_bytes = 0;
-    // small batches: split each (kernel, tree) task into R clock sub-ranges so that there are at
-    // least ~4 tasks per resident lane (R = 1 for large batches: every split costs an extra walk)
-    const long long lanes = (long long)sm_count(0) * 1024, tasks = std::max<long long>(1, n_k * tt);
-    int nsub = (int)std::min<long long>(2, std::max<long long>(1, (4 * lanes + tasks - 1) / tasks));
-    nsub = std::max(1, std::min(env_int("SYNERGY_NSUB", nsub), std::max(1, n_f)));
-    c.slots = nsub;                                        // carried to SweepArgs.nsub
-    c.smem = da_smem(nt, kpc, n_f, c.xs, nm);
-    while (c.smem > 200 * 1024 && c.tile_k > 1) c.smem = da_smem(nt, --c.tile_k, n_f, c.xs, nm);
-    c.head_bytes = (int)da_head(nt, c.tile_k, n_f, c.xs, nm);
-    return c.smem <= 200 * 1024;
-}
-
-template <int NT, bool TOPC>
-cudaError_t launch_da_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    static size_t smem_set = 48 * 1024;
-    if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep_da<NT, TOPC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
-        if (e != cudaSuccess) return e;
-        smem_set = c.smem;
-    }
-    k_sweep_da<NT, TOPC><<<(unsigned)grid, NT, c.smem, st>>>(a);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_da(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    const bool topc = da_topc();
-    if (c.nt == 256) return topc ? launch_da_t<256, true>(a, c, grid, st) : launch_da_t<256, false>(a, c, grid, st);
-    if (c.nt == 128) return topc ? launch_da_t<128, true>(a, c, grid, st) : launch_da_t<128, false>(a, c, grid, st);
-    return topc ? launch_da_t<64, true>(a, c, grid, st) : launch_da_t<64, false>(a, c, grid, st);
-}
-
 // ------------------------------------------------------------------ tree-major path (kernels_tm.cuh)
 // D difference arrays live in a library-owned buffer per (device, stream).  k_tm_finish zeroes
 // every entry it reads, so a buffer is all-zero between calls on its stream; a call that fails
-// after enqueuing k_tm_walk marks it dirty and the next call clears it with a memset.
+// after enqueuing k_tm_walk marks it dirty and the next call clears it with a memset.  Growing a
+// buffer is stream-ordered (pool free + alloc + memset on the caller's stream, no host sync).
 struct TmBuf {
     int dev;
     cudaStream_t st;
-    int kind;                        // 0/2: D and its second slab buffer (all-zero between calls), 1: k_tr_walk features
+    int kind;                        // 0 / 1: D and its second slab buffer
     long long* p;
     size_t bytes;
     bool dirty;
@@ -398,7 +318,7 @@ struct TmBuf {
 std::mutex g_tm_mu;
 std::list<TmBuf> g_tm_bufs;          // list: entries never move
 
-syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out, int kind = 0) {
+syn_status tm_buffer(DevState* ds, int dev, cudaStream_t st, size_t bytes, TmBuf** out, int kind) {
     std::lock_guard<std::mutex> lock(g_tm_mu);
     TmBuf* b = nullptr;
     for (TmBuf& x : g_tm_bufs)
@@ -409,22 +329,20 @@ syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out, int ki
     }
     cudaError_t e = cudaSuccess;
     if (b->bytes < bytes) {
-        if (b->p) {
-            cudaStreamSynchronize(st);          // the old buffer may still be read by queued work
-            cudaFree(b->p);
-            b->p = nullptr;
-            b->bytes = 0;
-        }
-        if ((e = cudaMalloc(&b->p, bytes)) != cudaSuccess) {
-            cudaGetLastError();
-            b->p = nullptr;
-            return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "tree-major D buffer of %zu bytes", bytes)
-                                                  : cuda_fail(e, "cudaMalloc(D)");
-        }
+        if (capturing(st))
+            return fail(SYN_ERR_UNSUPPORTED, "the sweep's scratch must grow inside a stream capture: call "
+                                             "synergy_prepare (or run one call of this shape) before capturing");
+        if (b->p) cudaFreeAsync(b->p, st);             // after the queued work on this stream
+        b->p = nullptr;
+        b->bytes = 0;
+        void* p = nullptr;
+        syn_status s = pool_alloc(ds, bytes, st, &p, "tree-major difference arrays");
+        if (s != SYN_OK) return s;
+        b->p = static_cast<long long*>(p);
         b->bytes = bytes;
         b->dirty = true;
     }
-    if (b->dirty && kind != 1) {
+    if (b->dirty) {
         if ((e = cudaMemsetAsync(b->p, 0, b->bytes, st)) != cudaSuccess) return cuda_fail(e, "cudaMemsetAsync(D)");
         b->dirty = false;
     }
@@ -434,7 +352,7 @@ syn_status tm_buffer(int dev, cudaStream_t st, size_t bytes, TmBuf** out, int ki
 
 // Slab pipeline (several kernel slabs per call): the finish of slab i runs on a library-owned
 // second stream while the walk of slab i + 1 runs on the caller's stream, with D double-buffered.
-// One side stream and three events per (device, caller stream).
+// One side stream and four events per (device, caller stream).
 struct TmAux {
     int dev;
     cudaStream_t st;
@@ -450,6 +368,9 @@ syn_status tm_aux(int dev, cudaStream_t st, TmAux** out) {
             *out = &x;
             return ok();
         }
+    if (capturing(st))
+        return fail(SYN_ERR_UNSUPPORTED, "slab-pipeline stream must be created before a stream capture: call "
+                                         "synergy_prepare (or run one call of this shape) first");
     TmAux x;
     x.dev = dev;
     x.st = st;
@@ -465,103 +386,108 @@ syn_status tm_aux(int dev, cudaStream_t st, TmAux** out) {
 }
 
 // Clock-cut copy of a model's blocks for one clock table (kernels_tm.cuh, k_cut_blocks), built on
-// first use and cached in the model.  The build is synchronous (once per model and table) so any
-// stream may use the copy afterwards.
+// first use on the caller's stream and cached in the model.  Later calls on another stream wait
+// for the build's event (until it is known complete); nothing synchronises the host.
 std::mutex g_cut_mu;
-syn_status cut_blocks(syn_model* m, const syn_clocks* c, const uint4** out) {
+syn_status cut_blocks(DevState* ds, syn_model* m, const syn_clocks* c, cudaStream_t st, const uint4** out) {
     std::lock_guard<std::mutex> lock(g_cut_mu);
-    for (auto& cb : m->cut_blocks)
-        if (cb.first == c->uid) {
-            *out = cb.second;
-            return ok();
+    for (CutCopy& cb : m->cuts) {
+        if (cb.uid != c->uid) continue;
+        if (cb.ready && !capturing(st)) {
+            const cudaError_t q = cudaEventQuery(cb.ready);
+            if (q == cudaSuccess) {
+                cudaEventDestroy(cb.ready);
+                cb.ready = nullptr;
+            } else if (q != cudaErrorNotReady) {
+                cudaGetLastError();
+            }
         }
-    uint4* p = nullptr;
-    const long long nb = std::max<long long>(m->n_blocks, 1);
-    cudaError_t e = cudaMalloc(&p, (size_t)nb * 2 * sizeof(uint4));
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return cuda_fail(e, "cudaMalloc(clock-cut blocks)");
+        if (cb.ready && cb.built_on != st) {
+            const cudaError_t e = cudaStreamWaitEvent(st, cb.ready, 0);
+            if (e != cudaSuccess) return cuda_fail(e, "wait for the clock-cut copy");
+        }
+        *out = cb.p;
+        return ok();
     }
-    if (m->n_blocks > 0)
-        k_cut_blocks<<<(unsigned)((m->n_blocks + 255) / 256), 256>>>(m->dm.blocks, m->n_blocks, m->n_inputs - 1,
-                                                                   c->d_freqs, c->n_f, m->dm.fx32 ? m->dm.fx_scale : 0.0, p);
-    if ((e = cudaGetLastError()) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess) {
-        cudaFree(p);
+    if (capturing(st))
+        return fail(SYN_ERR_UNSUPPORTED, "the clock-cut copy of a (model, clock table) pair must be built before a "
+                                         "stream capture: call synergy_prepare (or run one call) first");
+    void* p = nullptr;
+    const long long nb = std::max<long long>(m->n_blocks, 1);
+    syn_status s = pool_alloc(ds, (size_t)nb * 2 * sizeof(uint4), st, &p, "clock-cut blocks");
+    if (s != SYN_OK) return s;
+    cudaError_t e = cudaSuccess;
+    if (m->n_blocks > 0) {
+        KernelTimer kt("k_cut_blocks", st);
+        k_cut_blocks<<<(unsigned)((m->n_blocks + 255) / 256), 256, 0, st>>>(
+            m->dm.blocks, m->n_blocks, m->n_inputs - 1, c->d_freqs, c->n_f, m->dm.fx32 ? m->dm.fx_scale : 0.0,
+            static_cast<uint4*>(p));
+        e = cudaGetLastError();
+    }
+    cudaEvent_t ev = nullptr;
+    if (e == cudaSuccess && (e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) == cudaSuccess)
+        e = cudaEventRecord(ev, st);
+    if (e != cudaSuccess) {
+        cudaFreeAsync(p, st);
+        if (ev) cudaEventDestroy(ev);
         return cuda_fail(e, "k_cut_blocks");
     }
-    m->cut_blocks.push_back({c->uid, p});
-    *out = p;
+    m->cuts.push_back({c->uid, static_cast<uint4*>(p), st, ev});
+    *out = static_cast<const uint4*>(p);
     return ok();
 }
 
-// Tree-resident copy (kernels_tr.cuh, k_tr_layout) of a model's clock-cut blocks, cached like them.
-syn_status tr_blocks(syn_model* m, const syn_clocks* c, const uint4* cut, const uint4** out) {
-    std::lock_guard<std::mutex> lock(g_cut_mu);
-    for (auto& cb : m->tr_blocks)
-        if (cb.first == c->uid) {
-            *out = cb.second;
-            return ok();
-        }
-    uint4* p = nullptr;
-    const long long nb = std::max<long long>(m->n_blocks, 1);
-    cudaError_t e = cudaMalloc(&p, (size_t)nb * 2 * sizeof(uint4));
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return cuda_fail(e, "cudaMalloc(tree-resident blocks)");
-    }
-    if (m->n_trees > 0)
-        k_tr_layout<<<(unsigned)m->n_trees, 256>>>(cut, m->dm.broot, m->n_trees, m->n_blocks, p);
-    if ((e = cudaGetLastError()) != cudaSuccess || (e = cudaDeviceSynchronize()) != cudaSuccess) {
-        cudaFree(p);
-        return cuda_fail(e, "k_tr_layout");
-    }
-    m->tr_blocks.push_back({c->uid, p});
-    *out = p;
-    return ok();
+constexpr size_t kTmSlabBytes = 48u << 20;   // D bytes per slab (stays L2-resident with the model)
+
+const DevModel& dm_of(const SweepArgs& a, int m) { return m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2]; }
+bool present(const SweepArgs& a, int m) { return m < 2 || a.has_x[m - 2]; }
+
+size_t tm_walk_smem(int F, int tt) { return (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8; }
+size_t tm_finish_smem(int nm, int k, int n_f, int xs, int nslot) {
+    return (size_t)nm * k * n_f * 12 + (size_t)n_f * 4 + (size_t)k * xs * 4 + 32 + (size_t)k * nslot * n_f * 8;
 }
 
-constexpr size_t kTmSlabBytes = 48u << 20;
-constexpr size_t kTrTreeMax = 64u << 10;     // largest tree (bytes of 2-level blocks) k_tr_walk stages   // D bytes per slab (stays L2-resident with the model)
-
-// Tree-major path (k_tm_walk + k_tm_finish per kernel slab).  Needs every forest within the exact
-// int64 leaf range (fx_ok) and at least one tree; returns false (nothing enqueued) otherwise.
-bool tm_eligible(const SweepArgs& a, int nm) {
-    int tt = 0;
+// Tree-major path: needs every forest within the exact int64 leaf range (fx_ok), at least one
+// tree, and k_tm_walk / k_tm_finish within the device's shared memory.  Else the general path.
+bool tm_eligible(const SweepArgs& a, int nm, const DevState* ds) {
+    int tt = 0, nslot = 0;
     for (int m = 0; m < nm; ++m) {
-        if (m >= 2 && !a.has_x[m - 2]) continue;
-        const DevModel& d = m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+        if (!present(a, m)) continue;
+        const DevModel& d = dm_of(a, m);
         if (d.forest_weight == 0.0 || d.n_trees == 0) continue;
         if (!d.fx_ok) return false;
         tt += d.n_trees;
+        ++nslot;
     }
-    return tt > 0;
+    if (tt == 0) return false;
+    if (tm_walk_smem(a.F, tt) > (size_t)ds->optin) return false;
+    return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->optin;
+}
+
+int finish_ctas_per_sm(DevState* ds, int fnt, size_t smem) {
+    std::lock_guard<std::mutex> lock(ds->occ_mu);
+    for (auto& e : ds->finish_occ)
+        if (e.first == smem) return e.second;
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tm_finish, fnt, smem) != cudaSuccess) {
+        cudaGetLastError();
+        nb = 0;
+    }
+    ds->finish_occ.push_back({smem, nb});
+    return nb;
 }
 
 syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clocks* clocks, cudaStream_t st,
-                  int* launches, int* variant) {
+                  DevState* ds, bool prepare_only, int* launches) {
+    const Knobs& K = knobs();
     const int device = clocks->device;
     DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
-    // k_tm_walk (trees read through L1) by default; SYNERGY_TM_MODE=tr selects the tree-resident
-    // k_tr_walk when every tree fits its shared tree buffer (measured slower on the bench
-    // forests: with two 44-KB tree buffers per SM the lanes wait for stragglers)
-    const char* mode_env = getenv("SYNERGY_TM_MODE");
-    bool use_tr = mode_env && !strcmp(mode_env, "tr");
-    long long max_tb = 1;
-    for (int m = 0; m < nm; ++m)
-        if (models[m] && dms[m]->forest_weight != 0.0 && dms[m]->n_trees > 0)
-            max_tb = std::max(max_tb, models[m]->max_tree_blocks);
-    if ((size_t)max_tb * 32 > kTrTreeMax) use_tr = false;
-    for (int m = 0; m < nm; ++m)                  // k_tr_walk decodes int32 fixed-point leaves only
-        if (models[m] && dms[m]->forest_weight != 0.0 && dms[m]->n_trees > 0 && !dms[m]->fx32) use_tr = false;
-    TrArgs r;
-    memset(&r, 0, sizeof r);
     for (int m = 0; m < nm; ++m) {
         if (!models[m] || dms[m]->forest_weight == 0.0 || dms[m]->n_trees == 0) continue;
         const uint4* cb = nullptr;
-        syn_status cs = cut_blocks(models[m], clocks, &cb);
+        syn_status cs = cut_blocks(ds, models[m], clocks, st, &cb);
         if (cs != SYN_OK) return cs;
         dms[m]->blocks = cb;
-        if (use_tr && (cs = tr_blocks(models[m], clocks, cb, &r.trb[m])) != SYN_OK) return cs;
     }
     TmArgs t;
     memset(&t, 0, sizeof t);
@@ -571,8 +497,8 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     t.nslot = 0;
     for (int m = 0; m < 4; ++m) {
         t.slot_of[m] = -1;
-        if (m >= nm || (m >= 2 && !a.has_x[m - 2])) continue;
-        const DevModel& d = m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];
+        if (m >= nm || !present(a, m)) continue;
+        const DevModel& d = dm_of(a, m);
         if (d.forest_weight == 0.0 || d.n_trees == 0) continue;
         t.slot_of[m] = t.nslot++;
         tt += d.n_trees;
@@ -584,116 +510,67 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     // kernels per feature block: a power of two in [32, 256], F * kb floats of shared memory
     int kb = 256;
     while (kb > 32 && ((size_t)F * kb * 4 > 32768 || kb / 2 >= n_k)) kb /= 2;
-    const int kb_env = env_int("SYNERGY_TM_KB", kb);
-    while (kb > 32 && kb > kb_env) kb /= 2;
-    while (kb < 256 && kb * 2 <= kb_env) kb *= 2;
+    const long long kb_knob = K.tm_kb.load();
+    if (kb_knob > 0) {
+        while (kb > 32 && kb > kb_knob) kb /= 2;
+        while (kb < 256 && kb * 2 <= kb_knob) kb *= 2;
+    }
     t.kb = kb;
     t.kb_log2 = 0;
     while ((1 << t.kb_log2) < kb) ++t.kb_log2;
     const size_t row = (size_t)t.nslot * n_f * sizeof(long long);
     // kernels per slab: a multiple of the feature block, D of one slab <= kTmSlabBytes (L2-resident)
     long long nks = std::max<long long>(kb, (long long)(kTmSlabBytes / row) / kb * kb);
-    const int slab_env = env_int("SYNERGY_TM_SLAB", 0);
-    if (slab_env > 0) nks = std::max<long long>(kb, slab_env / kb * kb);
+    if (K.tm_slab.load() > 0) nks = std::max<long long>(kb, K.tm_slab.load() / kb * kb);
     nks = std::min<long long>(nks, n_k);
-    // k_tr_walk chunk size P (kernels per unit): 1024, halved down to 512 while that leaves fewer
-    // than 4 units per SM; the slab's transposed features ride in the same scratch as D
-    const int sms_tr = sm_count(device);
-    int P = 1024;
-    while (P > 512 && (long long)tt * ((std::min<long long>(nks, n_k) + P - 1) / P) < 4LL * sms_tr) P /= 2;
-    const int p_env = env_int("SYNERGY_TR_P", P);
-    if (p_env >= 32 && p_env <= 2048 && p_env % 32 == 0) P = p_env;
     TmBuf* buf = nullptr;
-    syn_status s = tm_buffer(device, st, (size_t)nks * row, &buf);
+    syn_status s = tm_buffer(ds, device, st, (size_t)nks * row, &buf, 0);
     if (s != SYN_OK) return s;
     t.D = buf->p;
     // several slabs: finish(i) on a side stream overlaps walk(i + 1); D alternates between two
     // buffers and walk(i + 2) waits for finish(i), which zeroes its buffer
-    const bool pipe = n_k > nks && env_int("SYNERGY_TM_PIPE", 1) != 0;
+    const bool pipe = n_k > nks && K.tm_pipe.load() != 0;
     TmBuf* buf2 = nullptr;
     TmAux* aux = nullptr;
     if (pipe) {
-        if ((s = tm_buffer(device, st, (size_t)nks * row, &buf2, 2)) != SYN_OK) return s;
+        if ((s = tm_buffer(ds, device, st, (size_t)nks * row, &buf2, 1)) != SYN_OK) return s;
         if ((s = tm_aux(device, st, &aux)) != SYN_OK) return s;
-    }
-    if (use_tr && F > 0) {
-        TmBuf* fb = nullptr;
-        if ((s = tm_buffer(device, st, (size_t)((nks + P - 1) / P) * F * P * 4, &fb, 1)) != SYN_OK) return s;
-        r.featT = reinterpret_cast<const float*>(fb->p);
     }
     // finish tile: KT kernels per CTA, fp64 + fp32 per (model, kernel, clock) in shared memory
     // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
-    int kt = std::max(1, std::min(8, (int)((150 * 1024) / ((size_t)nm * n_f * 12 + (size_t)t.nslot * n_f * 8))));
-    const int kt_cap = kt;                                         // shared-memory bound
     a.xs = (F + 2) | 1;
-    int fnt = env_int("SYNERGY_TM_FNT", 256);                     // finish CTA size
-    if (fnt != 128 && fnt != 256) fnt = 256;
-    auto fsmem_of = [&](int k) {
-        return (size_t)nm * k * n_f * 12 + (size_t)n_f * 4 + (size_t)k * a.xs * 4 + 32 + (size_t)k * t.nslot * n_f * 8;
-    };
-    static size_t fset = 48 * 1024, wset = 48 * 1024;
-    cudaError_t e = cudaSuccess;
-    if (fsmem_of(kt_cap) > fset) {
-        if ((e = cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem_of(kt_cap))) != cudaSuccess)
-            return cuda_fail(e, "k_tm_finish attribute");
-        fset = fsmem_of(kt_cap);
-    }
+    const int fnt = 256;
+    auto fsmem_of = [&](int k) { return tm_finish_smem(nm, k, n_f, a.xs, t.nslot); };
+    int kt_cap = 1;
+    while (kt_cap < 8 && fsmem_of(kt_cap + 1) <= std::min<size_t>((size_t)ds->optin, 150 * 1024)) ++kt_cap;
     // the smallest tile whose finish grid fits in one wave of resident CTAs (a partial second wave
     // doubles the finish's latency chain: c5 KT 3 -> 7 = 1195 -> 512 CTAs, 46 -> 37 us); when no
     // tile fits, the largest (kt_cap)
-    {
-        const int sms = sm_count(device);
-        int fit = 0;
-        for (int k = 1; k <= kt_cap && !fit; ++k) {
-            int nb = 0;
-            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tm_finish, fnt, fsmem_of(k)) != cudaSuccess) {
-                cudaGetLastError();
-                break;
-            }
-            if (nb > 0 && (nks + k - 1) / k <= (long long)nb * sms) fit = k;
-        }
-        kt = fit ? fit : kt_cap;
+    int kt = 0;
+    for (int k = 1; k <= kt_cap && !kt; ++k) {
+        const int nb = finish_ctas_per_sm(ds, fnt, fsmem_of(k));
+        if (nb > 0 && (nks + k - 1) / k <= (long long)nb * ds->sms) kt = k;
     }
-    kt = std::max(1, std::min(env_int("SYNERGY_TM_KT", kt), 8));
+    if (!kt) kt = kt_cap;
+    if (K.tm_kt.load() > 0) kt = (int)std::min<long long>(K.tm_kt.load(), kt_cap);
     a.tile_k = kt;
+    if (prepare_only) {                           // scratch, copies and the occupancy cache exist now
+        *launches = 0;
+        return ok();
+    }
     const size_t fsmem = fsmem_of(kt);
-    const size_t wsmem = (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8;
-    if (fsmem > fset) {
-        if ((e = cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)fsmem)) != cudaSuccess)
-            return cuda_fail(e, "k_tm_finish attribute");
-        fset = fsmem;
-    }
-    if (wsmem > wset) {
-        if ((e = cudaFuncSetAttribute(k_tm_walk<kTmNT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess ||
-            (e = cudaFuncSetAttribute(k_tm_walk<kTmNT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)wsmem)) != cudaSuccess)
-            return cuda_fail(e, "k_tm_walk attribute");
-        wset = wsmem;
-    }
-    static int carve_set = -1;                 // same shared-memory carveout for both kernels
-    const int carve = env_int("SYNERGY_TM_CARVE", -1);
-    if (carve != carve_set && carve >= 0) {
-        cudaFuncSetAttribute(k_tm_walk<kTmNT, true>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-        cudaFuncSetAttribute(k_tm_walk<kTmNT, false>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-        cudaFuncSetAttribute(k_tm_finish, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-        cudaGetLastError();
-        carve_set = carve;
-    }
-    const int ctas = std::max(1, env_int("SYNERGY_TM_CTAS", 2 * sm_count(device)));
-    // k_tr_walk: kTrNB tree buffers + the chunk's [F][P] features + record stacks
-    r.tree_smem = (int)(((size_t)max_tb * 32 + 127) / 128 * 128);
-    r.P = P;
-    const size_t rsmem = (size_t)kTrNB * r.tree_smem + (size_t)F * P * 4 + (size_t)kTmS * kTrNT * 8;
-    if (use_tr) {
-        static size_t rset = 48 * 1024;
-        if (rsmem > rset) {
-            if ((e = cudaFuncSetAttribute(k_tr_walk<kTrNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)rsmem)) != cudaSuccess)
-                return cuda_fail(e, "k_tr_walk attribute");
-            rset = rsmem;
-        }
-    }
+    const size_t wsmem = tm_walk_smem(F, tt);
+    const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : 2LL * ds->sms);
     t.s = a;
     int n = 0;
     int slab = 0;
+    cudaError_t e = cudaSuccess;
+    auto fail_launch = [&](const char* what) {
+        buf->dirty = true;
+        if (buf2) buf2->dirty = true;
+        if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
+        return cuda_fail(e, what);
+    };
     for (long long s0 = 0; s0 < n_k; s0 += nks, ++slab) {
         t.slab0 = s0;
         t.nks = (int)std::min<long long>(nks, n_k - s0);
@@ -701,7 +578,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         if (pipe) {
             t.D = pb ? buf2->p : buf->p;
             if (slab >= 2 && (e = cudaStreamWaitEvent(st, aux->finished[pb], 0)) != cudaSuccess)
-                return cuda_fail(e, "slab pipeline wait");
+                return fail_launch("slab pipeline wait");
         }
         // tiny batches: split every (kernel, tree) task into clock sub-ranges while there are fewer
         // tasks than resident lanes (at most 8 sub-ranges of at least 8 clocks; each sub-range
@@ -709,64 +586,30 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         t.nsub = 1;
         const long long lanes = (long long)ctas * kTmNT;
         while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8) t.nsub *= 2;
-        const int ns_env = env_int("SYNERGY_TM_NSUB", t.nsub);
-        if (ns_env >= 1 && ns_env <= n_f && ns_env <= 64) t.nsub = ns_env;
+        if (K.tm_nsub.load() >= 1 && K.tm_nsub.load() <= std::min(n_f, 64)) t.nsub = (int)K.tm_nsub.load();
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * t.nsub * kb;
         // a few tasks per lane: dynamic task fetch balances walks of different lengths
-        t.dyn = env_int("SYNERGY_TM_DYN", t.n_tasks < 4 * lanes ? 1 : 0) ? 1 : 0;
-        if (use_tr) {
-            // unit = (tree, chunk of P kernels), one CTA per SM over contiguous unit ranges
-            r.nchunks = (t.nks + P - 1) / P;
-            r.tm = t;
-            {
-                const long long nf = (long long)r.nchunks * F * P;
-                KernelTimer ktf("k_tr_feat", st);
-                if (nf > 0) k_tr_feat<<<(unsigned)((nf + 255) / 256), 256, 0, st>>>(a.features, t.slab0, t.nks, F, P, r.nchunks, const_cast<float*>(r.featT));
-                e = cudaGetLastError();
-            }
-            const long long units = (long long)r.nchunks * tt;
-            const long long g = std::max<long long>(1, std::min<long long>(env_int("SYNERGY_TR_CTAS", sms_tr), units));
-            if (e == cudaSuccess) {
-                KernelTimer ktm("k_tr_walk", st);
-                k_tr_walk<kTrNT><<<(unsigned)g, kTrNT, rsmem, st>>>(r);
-                e = cudaGetLastError();
-            }
-            if (e != cudaSuccess) {
-                buf->dirty = true;
-                if (buf2) buf2->dirty = true;
-                if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
-                return cuda_fail(e, "k_tr_walk launch");
-            }
-            ++n;
-        } else {
+        t.dyn = K.tm_dyn.load() >= 0 ? (K.tm_dyn.load() ? 1 : 0) : (t.n_tasks < 4 * lanes ? 1 : 0);
+        {
             const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
-            {
-                KernelTimer ktm("k_tm_walk", st);
-                if (fxall)
-                    k_tm_walk<kTmNT, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-                else
-                    k_tm_walk<kTmNT, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-                e = cudaGetLastError();
-            }
-            if (e != cudaSuccess) {
-                buf->dirty = true;
-                if (buf2) buf2->dirty = true;
-                if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
-                return cuda_fail(e, "k_tm_walk launch");
-            }
+            KernelTimer ktm("k_tm_walk", st);
+            if (fxall)
+                k_tm_walk<kTmNT, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            else
+                k_tm_walk<kTmNT, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            e = cudaGetLastError();
         }
+        if (e != cudaSuccess) return fail_launch("k_tm_walk launch");
         cudaStream_t fst = st;
         if (pipe) {
             if ((e = cudaEventRecord(aux->walked[pb], st)) != cudaSuccess ||
-                (e = cudaStreamWaitEvent(aux->st2, aux->walked[pb], 0)) != cudaSuccess) {
-                buf->dirty = buf2->dirty = true;
-                return cuda_fail(e, "slab pipeline fork");
-            }
+                (e = cudaStreamWaitEvent(aux->st2, aux->walked[pb], 0)) != cudaSuccess)
+                return fail_launch("slab pipeline fork");
             fst = aux->st2;
         }
         {
             KernelTimer ktm("k_tm_finish", fst);
-            if (!pipe && env_int("SYNERGY_TM_PDL", 1) != 0) {
+            if (!pipe && K.tm_pdl.load() != 0) {
                 // programmatic dependent launch: the finish grid is scheduled while the walk runs
                 // and waits (griddepcontrol.wait) for it before reading D
                 cudaLaunchConfig_t lc;
@@ -787,92 +630,67 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             }
         }
         if (e == cudaSuccess && pipe) e = cudaEventRecord(aux->finished[pb], aux->st2);
-        if (e != cudaSuccess) {
-            buf->dirty = true;
-            if (buf2) buf2->dirty = true;
-            if (pipe && slab > 0) cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0);
-            return cuda_fail(e, "k_tm_finish launch");
-        }
+        if (e != cudaSuccess) return fail_launch("k_tm_finish launch");
         n += 2;
     }
     if (pipe && (e = cudaStreamWaitEvent(st, aux->finished[(slab - 1) & 1], 0)) != cudaSuccess)   // join
         return cuda_fail(e, "slab pipeline join");
     *launches = n;
-    *variant = use_tr ? 4001 : 4000;
     return ok();
 }
 
-template <int S, int T>
-cudaError_t launch_sweep_t(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    static size_t smem_set = 48 * 1024;   // per-instantiation opt-in high-water mark
-    if (c.smem > smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_sweep<S, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.smem);
-        if (e != cudaSuccess) return e;
-        smem_set = c.smem;
-    }
-    k_sweep<S, T><<<(unsigned)grid, c.nt, c.smem, st>>>(a);
-    return cudaGetLastError();
-}
+// ---------------------------------------------------------- general exact path (kernels_gen.cuh)
+constexpr size_t kGenSlabBytes = 64u << 20;   // fp64 + fp32 scratch per kernel slab
 
-cudaError_t launch_sweep(const SweepArgs& a, const Config& c, long long grid, cudaStream_t st) {
-    switch (c.slots) {
-        case 1: return launch_sweep_t<1, 4>(a, c, grid, st);
-        case 2: return launch_sweep_t<2, 4>(a, c, grid, st);
-        case 4: return launch_sweep_t<4, 2>(a, c, grid, st);
-        default: return launch_sweep_t<8, 1>(a, c, grid, st);
-    }
-}
-
-syn_status validate_sweep(const syn_model* sp, const syn_model* en, int64_t n_k, int32_t F,
-                          const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t, int mode) {
-    if (!sp || !en) return fail(SYN_ERR_INVALID_ARG, "model is NULL");
-    if (!clocks) return fail(SYN_ERR_INVALID_ARG, "clocks is NULL");
-    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
-    if (F + 1 != sp->n_inputs || F + 1 != en->n_inputs)
-        return fail(SYN_ERR_INVALID_ARG, "n_features+1=%d does not match model n_inputs (%d, %d)", F + 1, sp->n_inputs, en->n_inputs);
-    const int n_f = clocks->n_f;
-    if (mode == kModeSweep) {
-        if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
-        syn_status s = check_targets(targets, n_t);
-        if (s != SYN_OK) return s;
-    } else if (def < -1 || def >= n_f) {
-        return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [-1, %d)", def, n_f);
-    }
-    if (sp->device != clocks->device || en->device != clocks->device || !current_device_is(clocks->device))
-        return fail(SYN_ERR_INVALID_ARG, "model/clocks device differs from the current device");
-    return SYN_OK;
-}
-
-// Library-owned stream-ordered pool per device for the SVR scratch: memory freed with
-// cudaFreeAsync stays mapped (release threshold = max), so steady-state calls reuse it instead
-// of remapping; the process's default pool and its settings are left alone.
-cudaMemPool_t svr_pool(int dev) {
-    static std::mutex mu;
-    static cudaMemPool_t pools[64] = {};
-    if (dev < 0 || dev >= 64) return nullptr;
-    std::lock_guard<std::mutex> lock(mu);
-    if (!pools[dev]) {
-        cudaMemPoolProps props;
-        memset(&props, 0, sizeof props);
-        props.allocType = cudaMemAllocationTypePinned;
-        props.handleTypes = cudaMemHandleTypeNone;
-        props.location.type = cudaMemLocationTypeDevice;
-        props.location.id = dev;
-        cudaMemPool_t p = nullptr;
-        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) {
-            cudaGetLastError();
-            return nullptr;
+syn_status run_gen(SweepArgs a, int nm, cudaStream_t st, DevState* ds, int* launches) {
+    const Knobs& K = knobs();
+    const int n_f = a.n_f;
+    const long long n_k = a.n_k;
+    const size_t per_kernel = (size_t)nm * n_f * 12;
+    long long nks = std::max<long long>(1, (long long)(kGenSlabBytes / per_kernel));
+    nks = std::min<long long>(nks, n_k);
+    int kt = (int)std::max<long long>(1, std::min<long long>(8, nks / (2LL * ds->sms)));
+    if (K.gen_kt.load() > 0) kt = (int)std::min<long long>(K.gen_kt.load(), 64);
+    a.tile_k = kt;
+    void* scr = nullptr;
+    const size_t mvb = (size_t)nks * per_kernel / 12 * 8;
+    syn_status s = pool_alloc(ds, (size_t)nks * per_kernel + 256, st, &scr, "general-path scratch");
+    if (s != SYN_OK) return s;
+    GenArgs g;
+    memset(&g, 0, sizeof g);
+    g.s = a;
+    g.mv = static_cast<double*>(scr);
+    g.sv = reinterpret_cast<float*>(static_cast<char*>(scr) + (mvb + 255) / 256 * 256);
+    g.nm = nm;
+    int n = 0;
+    cudaError_t e = cudaSuccess;
+    for (long long s0 = 0; s0 < n_k && e == cudaSuccess; s0 += nks) {
+        g.slab0 = s0;
+        g.nks = (int)std::min<long long>(nks, n_k - s0);
+        const long long units = (long long)g.nks * n_f;
+        {
+            KernelTimer kt1("k_gen_forest", st);
+            k_gen_forest<<<(unsigned)((units + 255) / 256), 256, 0, st>>>(g);
+            e = cudaGetLastError();
         }
-        unsigned long long thr = ~0ULL;
-        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
-        pools[dev] = p;
+        if (e != cudaSuccess) break;
+        {
+            KernelTimer kt2("k_gen_finish", st);
+            k_gen_finish<<<(unsigned)((g.nks + kt - 1) / kt), 256, 0, st>>>(g);
+            e = cudaGetLastError();
+        }
+        n += 2;
     }
-    return pools[dev];
+    cudaFreeAsync(scr, st);
+    if (e != cudaSuccess) return cuda_fail(e, "general-path launch");
+    *launches = n;
+    return ok();
 }
 
+// ------------------------------------------------------------------------ SVR member
 // SVR members (kernels_svr.cuh): per model, V = clock factors and the split contractions P into
-// stream-ordered scratch; dm.svr_p / svr_splits point the finish step at them.  Released with
-// release() after the sweep kernel is enqueued (cudaFreeAsync keeps it alive until then).
+// stream-ordered scratch from the library pool; dm.svr_p / svr_splits point the finish step at
+// them.  Released (cudaFreeAsync) after the sweep's kernels are enqueued.
 struct SvrScratch {
     std::vector<void*> bufs;
     cudaStream_t st = nullptr;
@@ -886,20 +704,14 @@ struct SvrScratch {
 
 template <int CPT>
 cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, cudaStream_t st) {
-    static bool smem_set = false;
     const size_t smem = (size_t)kSvrStages * kSvrJC * (kSvrTK + 32 * CPT) * sizeof(double) + kSvrStages * 8;
-    if (!smem_set) {
-        cudaError_t e = cudaFuncSetAttribute(k_svr<CPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        smem_set = true;
-    }
     k_svr<CPT><<<grid, 256, smem, st>>>(sa);
     return cudaGetLastError();
 }
 
 constexpr size_t kSvrSlabBytes = 256u << 20;   // U scratch per kernel slab
 
-syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
+syn_status prepare_svr(DevModel& dm, DevState* ds, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
                        cudaStream_t st, SvrScratch& scr) {
     if (dm.svr_weight == 0.0) return ok();
     scr.st = st;
@@ -915,9 +727,9 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     const long long tiles = (std::min(nks, n_k) + kSvrTK - 1) / kSvrTK * tiles_n;
     if ((nks + kSvrTK - 1) / kSvrTK > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for k_svr");
     // split the SV range across CTAs until the grid covers the SMs (at most kSvrMaxSplits)
-    int splits = (int)std::max<long long>(1, sm_count(device) / std::max<long long>(tiles, 1));
+    int splits = (int)std::max<long long>(1, ds->sms / std::max<long long>(tiles, 1));
     splits = std::min(splits, kSvrMaxSplits);
-    splits = env_int("SYNERGY_SVR_SPLITS", splits);
+    if (knobs().svr_splits.load() > 0) splits = (int)std::min<long long>(knobs().svr_splits.load(), kSvrMaxSplits);
     splits = std::max(1, std::min(splits, n_chunks));
     const int cps = (n_chunks + splits - 1) / splits;
     splits = (n_chunks + cps - 1) / cps;
@@ -927,14 +739,8 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     const size_t voff = (pb + 255) / 256 * 256, uoff = voff + (vb + 255) / 256 * 256;
     const size_t total = uoff + ub;
     void* buf = nullptr;
-    cudaMemPool_t pool = svr_pool(device);
-    if (!pool) return fail(SYN_ERR_CUDA, "cannot create the SVR scratch pool on device %d", device);
-    cudaError_t e = cudaMallocFromPoolAsync(&buf, total, pool, st);
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return e == cudaErrorMemoryAllocation ? fail(SYN_ERR_OOM, "SVR scratch of %zu bytes", total)
-                                              : cuda_fail(e, "cudaMallocFromPoolAsync(SVR scratch)");
-    }
+    syn_status ps = pool_alloc(ds, total, st, &buf, "SVR scratch");
+    if (ps != SYN_OK) return ps;
     scr.bufs.push_back(buf);
     SvrArgs sa;
     memset(&sa, 0, sizeof sa);
@@ -956,6 +762,7 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     sa.Vt = reinterpret_cast<double*>(static_cast<char*>(buf) + voff);
     sa.Ut = reinterpret_cast<double*>(static_cast<char*>(buf) + uoff);
     const long long nv = (long long)tiles_n * n_svp * tn;
+    cudaError_t e;
     {
         KernelTimer kt("k_svr_v", st);
         k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
@@ -963,13 +770,8 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     }
     if (e != cudaSuccess) return cuda_fail(e, "k_svr_v launch");
     scr.launches += 1;
-    static bool u_smem_set = false;
     const size_t usmem = (size_t)F * (64 * sizeof(double) + kSvrJC * sizeof(float));
-    if (usmem > 48 * 1024 && !u_smem_set) {
-        if ((e = cudaFuncSetAttribute(k_svr_u, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024)) != cudaSuccess)
-            return cuda_fail(e, "k_svr_u attribute");
-        u_smem_set = true;
-    }
+    if (usmem > (size_t)ds->optin) return fail(SYN_ERR_UNSUPPORTED, "SVR member with %d inputs exceeds shared memory", F + 1);
     for (long long s0 = 0; s0 < n_k; s0 += nks) {
         sa.slab0 = s0;
         sa.nks = (int)std::min<long long>(nks, n_k - s0);
@@ -1000,101 +802,102 @@ syn_status prepare_svr(DevModel& dm, int device, const float* d_features, long l
     return ok();
 }
 
-syn_status run_sweep(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
-                     int32_t F, const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
-                     int32_t* d_choice, float* d_S, float* d_E, int mode, cudaStream_t st) {
-    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, mode);
+// --------------------------------------------------------------------- sweep driver
+
+syn_status validate_models(const syn_model* const* models, int nm, int32_t F, const syn_clocks* clocks) {
+    if (!models[0] || !models[1]) return fail(SYN_ERR_INVALID_ARG, "model is NULL");
+    if (!clocks) return fail(SYN_ERR_INVALID_ARG, "clocks is NULL");
+    for (int m = 0; m < nm; ++m) {
+        const syn_model* x = models[m];
+        if (!x) continue;
+        if (F + 1 != x->n_inputs)
+            return fail(SYN_ERR_INVALID_ARG, "n_features+1=%d does not match model %d n_inputs=%d", F + 1, m, x->n_inputs);
+        if (x->device != clocks->device) return fail(SYN_ERR_INVALID_ARG, "model %d / clocks on different devices", m);
+    }
+    if (!current_device_is(clocks->device)) return fail(SYN_ERR_INVALID_ARG, "clocks device differs from the current device");
+    return SYN_OK;
+}
+
+// One predict / sweep / sweep4 call.  models[0..1] speedup, energy; models[2..3] (nm == 4) direct
+// EDP / ED2P or NULL.  pred[m] = output planes or NULL.
+syn_status run_sweep(const syn_model* const* models, int nm, const float* d_features, int64_t n_k, int32_t F,
+                     const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
+                     int32_t* d_choice, float* const* pred, int mode, cudaStream_t st, bool prepare_only = false) {
+    syn_status vs = validate_models(models, nm, F, clocks);
     if (vs != SYN_OK) return vs;
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
     const int n_f = clocks->n_f;
+    if (mode == kModeSweep) {
+        if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
+        if (!prepare_only) {
+            vs = check_targets(targets, n_t);
+            if (vs != SYN_OK) return vs;
+        }
+    } else if (def < -1 || def >= n_f) {
+        return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [-1, %d)", def, n_f);
+    }
     if (n_k == 0) {
         g_last = {0, 0, 0, 0, 0};
         return ok();
     }
-    if (!d_features) return fail(SYN_ERR_INVALID_ARG, "d_features is NULL");
-    if (mode == kModeSweep && !d_choice) return fail(SYN_ERR_INVALID_ARG, "d_choice is NULL");
-    if (mode == kModePredict && (!d_S || !d_E)) return fail(SYN_ERR_INVALID_ARG, "d_speedup/d_energy is NULL");
+    if (!prepare_only) {
+        if (!d_features) return fail(SYN_ERR_INVALID_ARG, "d_features is NULL");
+        if (mode == kModeSweep && !d_choice) return fail(SYN_ERR_INVALID_ARG, "d_choice is NULL");
+        if (mode == kModePredict && (!pred[0] || !pred[1])) return fail(SYN_ERR_INVALID_ARG, "d_speedup/d_energy is NULL");
+    }
+    if ((n_k + 7) / 8 > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one call");
+    DevState* ds = nullptr;
+    if ((vs = need_dev(clocks->device, &ds)) != SYN_OK) return vs;
 
     SweepArgs a;
     memset(&a, 0, sizeof a);
-    a.ms = sp->dm;
-    a.me = en->dm;
+    a.ms = models[0]->dm;
+    a.me = models[1]->dm;
+    for (int x = 0; x < 2; ++x)
+        if (nm > 2 + x && models[2 + x]) {
+            a.mx[x] = models[2 + x]->dm;
+            a.has_x[x] = 1;
+        }
     a.features = d_features;
     a.n_k = n_k;
     a.F = F;
     a.freqs = clocks->d_freqs;
     a.n_f = n_f;
     a.def = def;
-    a.n_t = mode == kModeSweep ? n_t : 0;
+    a.n_t = mode == kModeSweep && !prepare_only ? n_t : 0;
     for (int t = 0; t < a.n_t; ++t) {
         a.kind[t] = targets[t].kind;
         a.x[t] = targets[t].x;
     }
     a.choice = d_choice;
-    a.S_out = d_S;
-    a.E_out = d_E;
+    a.S_out = pred[0];
+    a.E_out = pred[1];
+    a.X_out[0] = nm > 2 ? pred[2] : nullptr;
+    a.X_out[1] = nm > 3 ? pred[3] : nullptr;
     a.mode = mode;
-    // default: clock-interval traversal when forests are present and n_f <= 1024;
-    // SYNERGY_ALGO=direct forces the per-clock root-to-leaf kernel (A/B and fallback)
-    const char* algo_env = getenv("SYNERGY_ALGO");
-    const bool force_direct = algo_env && !strcmp(algo_env, "direct");
-    const bool force_iv = algo_env && !strcmp(algo_env, "iv");
-    const bool force_ws = algo_env && !strcmp(algo_env, "ws");
-    Config c;
-    const bool forests = sp->n_trees > 0 || en->n_trees > 0;
-    // default: order-free difference-array kernel (exact int64 leaf sums; n_f <= 2048), else the
-    // in-order warp-streaming kernel (n_f <= 256), else the chunked interval kernel
-    // (n_f <= 1024), else per-clock direct traversal; SYNERGY_ALGO=ws|iv|direct forces one
-    bool chosen = false;
-    if (!force_direct && forests) {
-        if (!force_iv && !force_ws) chosen = choose_da(sp, en, n_k, n_f, F, c);
-        if (!chosen && !force_iv) chosen = choose_ws(n_k, n_f, F, clocks->device, c);
-        if (!chosen) chosen = choose_iv(n_k, n_f, F, clocks->device, c);
-    }
-    if (!chosen) c = choose_config(n_k, n_f, F, clocks->device);
-    a.tile_k = c.tile_k;
-    a.xs = c.xs;
-    a.tc = c.tc;
-    a.words = c.words;
-    a.vcap = c.vcap;
-    a.vs = c.vs;
-    a.region = c.region;
-    a.win = c.win;
-    a.slot_bytes = c.slot_bytes;
-    a.head_bytes = c.head_bytes;
-    a.grid = clocks->d_grid;
-    a.f0 = clocks->f0;
-    a.inv_step = clocks->inv_step;
-    a.nsub = c.algo == 3 ? c.slots : 1;
-    const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
-    if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    SvrScratch scr;
-    syn_status ss = prepare_svr(a.ms, clocks->device, d_features, n_k, F, clocks, st, scr);
-    if (ss == SYN_OK) ss = prepare_svr(a.me, clocks->device, d_features, n_k, F, clocks, st, scr);
-    if (ss != SYN_OK) return ss;
-    // default: tree-major resume walks (kernels_tm.cuh) whenever the exact int64 leaf sums apply;
-    // SYNERGY_ALGO=da|ws|iv|direct selects one of the single-launch kernels instead
-    if (!algo_env && tm_eligible(a, 2)) {
+    a.xs = (F + 2) | 1;
+    const bool tm = knobs().algo.load() == 0 && tm_eligible(a, nm, ds);
+    if (prepare_only) {
+        if (!tm) return ok();
         int nl = 0;
-        syn_model* ms[2] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en)};
-        int var = 4000;
-        ss = run_tm(a, 2, ms, clocks, st, &nl, &var);
+        return run_tm(a, nm, const_cast<syn_model* const*>(models), clocks, st, ds, true, &nl);
+    }
+    SvrScratch scr;
+    DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
+    syn_status ss = SYN_OK;
+    for (int m = 0; m < nm && ss == SYN_OK; ++m)
+        if (present(a, m)) ss = prepare_svr(*dms[m], ds, d_features, n_k, F, clocks, st, scr);
+    if (ss != SYN_OK) return ss;
+    int nl = 0;
+    if (tm) {
+        ss = run_tm(a, nm, const_cast<syn_model* const*>(models), clocks, st, ds, false, &nl);
         if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k),
-                  var == 4001 ? kTrNT : kTmNT, var};
+        g_last = {nl + scr.launches, n_k * (long long)n_f, std::min<long long>(2LL * ds->sms, n_k), kTmNT, kVarTm};
         return ok();
     }
-    static const char* knames[4] = {"k_sweep", "k_sweep_iv", "k_sweep_ws", "k_sweep_da"};
-    cudaError_t e;
-    {
-        KernelTimer kt(knames[c.algo], st);
-        e = c.algo == 3 ? launch_da(a, c, grid, st)
-                  : c.algo == 2 ? launch_ws(a, c, grid, st)
-                  : c.algo == 1 ? launch_iv(a, c, grid, st)
-                                : launch_sweep(a, c, grid, st);
-    }
-    static const char* names[4] = {"k_sweep launch", "k_sweep_iv launch", "k_sweep_ws launch", "k_sweep_da launch"};
-    if (e != cudaSuccess) return cuda_fail(e, names[c.algo]);
-    g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, c.algo ? c.algo * 1000 + c.tile_k : c.slots * 10 + c.tilp};
+    ss = run_gen(a, nm, st, ds, &nl);
+    if (ss != SYN_OK) return ss;
+    g_last = {nl + scr.launches, n_k * (long long)n_f, ((long long)n_k * n_f + 255) / 256, 256, kVarGen};
     return ok();
 }
 
@@ -1107,6 +910,28 @@ extern "C" {
 const char* synergy_last_error(void) { return g_err.c_str(); }
 
 int32_t synergy_version(void) { return SYNERGY_VERSION; }
+
+syn_status synergy_config_set(const char* key, int64_t value) {
+    if (!key) return fail(SYN_ERR_INVALID_ARG, "key is NULL");
+    knobs();
+    for (const KnobName& k : kKnobs)
+        if (!strcmp(k.name, key)) {
+            k.v->store(value);
+            return ok();
+        }
+    return fail(SYN_ERR_INVALID_ARG, "unknown tuning key '%s'", key);
+}
+
+syn_status synergy_config_get(const char* key, int64_t* value) {
+    if (!key || !value) return fail(SYN_ERR_INVALID_ARG, "key/value is NULL");
+    knobs();
+    for (const KnobName& k : kKnobs)
+        if (!strcmp(k.name, key)) {
+            *value = k.v->load();
+            return ok();
+        }
+    return fail(SYN_ERR_INVALID_ARG, "unknown tuning key '%s'", key);
+}
 
 syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_model** out) {
     if (!out) return fail(SYN_ERR_INVALID_ARG, "out is NULL");
@@ -1168,6 +993,9 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
                 memcpy(&vb, &v, 4);
                 depth = std::max(depth, qdepth[p]);
                 if (f < 0) {
+                    // leaves must be finite: the exact sums (Q8) are defined on reals
+                    if (!std::isfinite(v))
+                        return fail(SYN_ERR_INVALID_ARG, "tree %d node %lld: leaf value is not finite", t, (long long)id);
                     nodes.push_back(make_uint2(vb, 0xFFFFFF00u | leaf_code));
                     continue;
                 }
@@ -1191,35 +1019,30 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
             max_depth = std::max(max_depth, depth);
         }
     }
-    // exact fixed-point scale for the leaf sums (k_sweep_da): s = -(smallest leaf ulp exponent)
+    // exact fixed-point scale for the leaf sums: s = -(smallest leaf ulp exponent); fx_ok when
+    // T * max|v| * 2^s < 2^62 (one int64), fx32 when every |v| * 2^s < 2^31
     int fx_ok = 0, fx_s = 0, fx32 = 0;
     if (d->forest_weight != 0.0) {
         int min_lsb = 1 << 30, max_e = -(1 << 30);
-        bool finite = true;
-        for (int t = 0; t < d->n_trees && finite; ++t)
-            for (int64_t id = d->tree_offset[t]; id < d->tree_offset[t + 1]; ++id) {
-                if (d->feature[id] >= 0) continue;
-                const float v = d->value[id];
-                if (!std::isfinite(v)) { finite = false; break; }
-                if (v == 0.0f) continue;
-                int e2 = 0;
-                std::frexp(v, &e2);                       // |v| in [2^(e2-1), 2^e2)
-                min_lsb = std::min(min_lsb, std::max(e2 - 24, -149));
-                max_e = std::max(max_e, e2);
-            }
-        if (finite) {
-            if (max_e == -(1 << 30)) { fx_ok = 1; fx_s = 0; fx32 = 1; }   // all leaves zero
-            else {
-                fx_s = -min_lsb;
-                int lg = 0;
-                while ((1LL << lg) < (long long)d->n_trees + 1) ++lg;
-                fx_ok = (max_e + fx_s + lg <= 61) ? 1 : 0;
-                fx32 = (fx_ok && max_e + fx_s <= 31) ? 1 : 0;
-            }
+        for (const uint2& nd : nodes) {
+            if ((nd.y & 0xffu) != leaf_code) continue;
+            float v;
+            memcpy(&v, &nd.x, 4);
+            if (v == 0.0f) continue;
+            int e2 = 0;
+            std::frexp(v, &e2);                       // |v| in [2^(e2-1), 2^e2)
+            min_lsb = std::min(min_lsb, std::max(e2 - 24, -149));
+            max_e = std::max(max_e, e2);
+        }
+        if (max_e == -(1 << 30)) { fx_ok = 1; fx_s = 0; fx32 = 1; }   // all leaves zero
+        else {
+            fx_s = -min_lsb;
+            int lg = 0;
+            while ((1LL << lg) < (long long)d->n_trees + 1) ++lg;
+            fx_ok = (max_e + fx_s + lg <= 61) ? 1 : 0;
+            fx32 = (fx_ok && max_e + fx_s <= 31) ? 1 : 0;
         }
     }
-    const int pad_leaf = (int)nodes.size();
-    nodes.push_back(make_uint2(0u, 0xFFFFFF00u | leaf_code));
 
     // 2-level blocks (see internal.h): built from the validated description, breadth-first
     std::vector<uint4> blocks;
@@ -1280,7 +1103,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
 
     DeviceGuard g(device);
     if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
-    const size_t nb = nodes.size() * sizeof(uint2);
+    const size_t nb = std::max<size_t>(nodes.size(), 1) * sizeof(uint2);
     const size_t tb = std::max<size_t>(trees.size(), 1) * sizeof(int2);
     const size_t lb = (size_t)d->n_inputs * sizeof(double);
     const size_t bb = std::max<size_t>(blocks.size(), 2) * sizeof(uint4);
@@ -1298,7 +1121,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     char* base = static_cast<char*>(mem);
     std::vector<double> lw((size_t)d->n_inputs, 0.0);
     if (d->linear_weight != 0.0) std::copy(d->lin_w, d->lin_w + d->n_inputs, lw.begin());
-    if ((e = cudaMemcpy(base, nodes.data(), nb, cudaMemcpyHostToDevice)) != cudaSuccess ||
+    if ((!nodes.empty() && (e = cudaMemcpy(base, nodes.data(), nodes.size() * sizeof(uint2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (!trees.empty() && (e = cudaMemcpy(base + off_t, trees.data(), trees.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
         (!blocks.empty() && (e = cudaMemcpy(base + off_b, blocks.data(), blocks.size() * sizeof(uint4), cudaMemcpyHostToDevice)) != cudaSuccess) ||
@@ -1320,7 +1143,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->n_inputs = d->n_inputs;
     m->n_trees = d->forest_weight != 0.0 ? d->n_trees : 0;
     m->max_depth = max_depth;
-    m->n_nodes = (long long)nodes.size() - 1;
+    m->n_nodes = (long long)nodes.size();
     m->bytes = (long long)total;
     m->alloc = mem;
     m->dm.nodes = reinterpret_cast<const uint2*>(base);
@@ -1330,19 +1153,15 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.lin_weight = d->linear_weight;
     m->dm.forest_weight = d->forest_weight;
     m->dm.n_trees = m->n_trees;
-    m->dm.pad_leaf = pad_leaf;
     m->dm.depth = max_depth;
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
     m->dm.bdepth = bdepth;
     m->n_blocks = (long long)(blocks.size() >> 1);
     m->dm.nblk = (int)m->n_blocks;
-    m->max_tree_blocks = 0;
-    for (size_t t = 0; t < broot.size(); ++t)
-        m->max_tree_blocks = std::max<long long>(m->max_tree_blocks,
-                                                 (t + 1 < broot.size() ? broot[t + 1] : m->n_blocks) - broot[t]);
     m->dm.fx_ok = fx_ok;
     m->dm.fx32 = fx32;
+    m->dm.fx_s = fx_s;
     m->dm.fx_scale = std::ldexp(1.0, fx_s);
     m->dm.fx_inv = std::ldexp(1.0, -fx_s);
     m->dm.svr_weight = d->svr_weight;
@@ -1365,9 +1184,14 @@ syn_status synergy_model_destroy(syn_model* m) {
     if (!m) return ok();
     {
         DeviceGuard g(m->device);
+        cudaDeviceSynchronize();           // no queued work may still read the model's copies
         cudaFree(m->alloc);
-        for (auto& cb : m->cut_blocks) cudaFree(cb.second);
-        for (auto& cb : m->tr_blocks) cudaFree(cb.second);
+        for (CutCopy& cb : m->cuts) {
+            cudaFreeAsync(cb.p, nullptr);
+            if (cb.ready) cudaEventDestroy(cb.ready);
+        }
+        cudaStreamSynchronize(nullptr);
+        cudaGetLastError();
     }
     delete m;
     return ok();
@@ -1395,22 +1219,10 @@ syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, sy
         if (!(h[i - 1] < h[i])) return fail(SYN_ERR_INVALID_ARG, "freqs not strictly ascending at %d", i);
     DeviceGuard g(device);
     if (!g.okay) return fail(SYN_ERR_INVALID_ARG, "cannot select device %d", device);
-    // clock-cut hint grid: grid[b] = #{i : f_i < f_0 + b * step}, b = 0..kGrid (any rounding is
-    // fine: the kernels finish every cut with exact comparisons against the table)
-    const float f0 = h[0], span = h[n_f - 1] - h[0];
-    const float step = span > 0.0f ? span / (float)kGrid : 1.0f;
-    std::vector<unsigned short> grid(kGrid + 1);
-    for (int b = 0; b <= kGrid; ++b) {
-        const float edge = f0 + (float)b * step;
-        grid[b] = (unsigned short)(std::lower_bound(h, h + n_f, edge) - h);
-    }
     float* d = nullptr;
-    const size_t gbytes = (size_t)(kGrid + 1) * sizeof(unsigned short);
-    const size_t goff = ((size_t)n_f * sizeof(float) + 255) / 256 * 256;
-    cudaError_t e = cudaMalloc(&d, goff + gbytes);
+    cudaError_t e = cudaMalloc(&d, (size_t)n_f * sizeof(float));
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(clocks)");
-    if ((e = cudaMemcpy(d, h, (size_t)n_f * sizeof(float), cudaMemcpyHostToDevice)) != cudaSuccess ||
-        (e = cudaMemcpy(reinterpret_cast<char*>(d) + goff, grid.data(), gbytes, cudaMemcpyHostToDevice)) != cudaSuccess) {
+    if ((e = cudaMemcpy(d, h, (size_t)n_f * sizeof(float), cudaMemcpyHostToDevice)) != cudaSuccess) {
         cudaFree(d);
         return cuda_fail(e, "cudaMemcpy(clocks)");
     }
@@ -1422,9 +1234,6 @@ syn_status synergy_clocks_create(const float* h, int32_t n_f, int32_t device, sy
     c->device = device;
     c->n_f = n_f;
     c->d_freqs = d;
-    c->d_grid = reinterpret_cast<unsigned short*>(reinterpret_cast<char*>(d) + goff);
-    c->f0 = f0;
-    c->inv_step = 1.0f / step;
     static std::atomic<long long> next_uid{1};
     c->uid = next_uid++;
     *out = c;
@@ -1447,17 +1256,30 @@ syn_status synergy_clocks_info(const syn_clocks* c, int32_t* n_freqs) {
     return ok();
 }
 
+syn_status synergy_prepare(const syn_model* const* models, int32_t n_models, int64_t n_kernels, int32_t n_features,
+                           const syn_clocks* clocks, syn_stream stream) {
+    if (!models) return fail(SYN_ERR_INVALID_ARG, "models is NULL");
+    if (n_models != 2 && n_models != 4) return fail(SYN_ERR_INVALID_ARG, "n_models=%d (2 or 4)", n_models);
+    float* pred[4] = {nullptr, nullptr, nullptr, nullptr};
+    return run_sweep(models, n_models, nullptr, n_kernels, n_features, clocks, 0, nullptr, 0, nullptr, pred,
+                     kModeSweep, static_cast<cudaStream_t>(stream), true);
+}
+
 syn_status synergy_predict(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
                            int32_t F, const syn_clocks* clocks, int32_t def, float* d_S, float* d_E,
                            syn_stream stream) {
-    return run_sweep(sp, en, d_features, n_k, F, clocks, def, nullptr, 0, nullptr, d_S, d_E, kModePredict,
+    const syn_model* models[2] = {sp, en};
+    float* pred[4] = {d_S, d_E, nullptr, nullptr};
+    return run_sweep(models, 2, d_features, n_k, F, clocks, def, nullptr, 0, nullptr, pred, kModePredict,
                      static_cast<cudaStream_t>(stream));
 }
 
 syn_status synergy_sweep(const syn_model* sp, const syn_model* en, const float* d_features, int64_t n_k,
                          int32_t F, const syn_clocks* clocks, int32_t def, const syn_target* targets,
                          int32_t n_t, int32_t* d_choice, float* d_S, float* d_E, syn_stream stream) {
-    return run_sweep(sp, en, d_features, n_k, F, clocks, def, targets, n_t, d_choice, d_S, d_E, kModeSweep,
+    const syn_model* models[2] = {sp, en};
+    float* pred[4] = {d_S, d_E, nullptr, nullptr};
+    return run_sweep(models, 2, d_features, n_k, F, clocks, def, targets, n_t, d_choice, pred, kModeSweep,
                      static_cast<cudaStream_t>(stream));
 }
 
@@ -1465,89 +1287,16 @@ syn_status synergy_sweep4(const syn_model* const* models, const float* d_feature
                           const syn_clocks* clocks, int32_t def, const syn_target* targets, int32_t n_t,
                           int32_t* d_choice, float* d_pred, syn_stream stream) {
     if (!models) return fail(SYN_ERR_INVALID_ARG, "models is NULL");
-    const syn_model* sp = models[0];
-    const syn_model* en = models[1];
-    const syn_model* x2 = models[2];
-    const syn_model* x3 = models[3];
-    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, kModeSweep);
-    if (vs != SYN_OK) return vs;
-    for (const syn_model* xm : {x2, x3}) {
-        if (!xm) continue;
-        if (xm->n_inputs != F + 1) return fail(SYN_ERR_INVALID_ARG, "direct EDP/ED2P model n_inputs mismatch");
-        if (xm->device != clocks->device) return fail(SYN_ERR_INVALID_ARG, "model device differs from clocks");
+    float* pred[4] = {nullptr, nullptr, nullptr, nullptr};
+    if (d_pred && n_k > 0 && clocks) {
+        const size_t plane = (size_t)n_k * clocks->n_f;
+        pred[0] = d_pred;
+        pred[1] = d_pred + plane;
+        pred[2] = models[2] ? d_pred + 2 * plane : nullptr;
+        pred[3] = models[3] ? d_pred + 3 * plane : nullptr;
     }
-    if (n_k == 0) {
-        g_last = {0, 0, 0, 0, 0};
-        return ok();
-    }
-    if (!d_features || !d_choice) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
-    const int n_f = clocks->n_f;
-    Config c;
-    if (!choose_da(sp, en, n_k, n_f, F, c, x2, x3))
-        return fail(SYN_ERR_UNSUPPORTED, "four-model sweep needs forests within the exact int64 leaf range and n_freqs <= 2048");
-    SweepArgs a;
-    memset(&a, 0, sizeof a);
-    a.ms = sp->dm;
-    a.me = en->dm;
-    if (x2) { a.mx[0] = x2->dm; a.has_x[0] = 1; }
-    if (x3) { a.mx[1] = x3->dm; a.has_x[1] = 1; }
-    if (!x2 && !x3) a.has_x[0] = 0;
-    a.features = d_features;
-    a.n_k = n_k;
-    a.F = F;
-    a.freqs = clocks->d_freqs;
-    a.n_f = n_f;
-    a.def = def;
-    a.n_t = n_t;
-    for (int t = 0; t < n_t; ++t) {
-        a.kind[t] = targets[t].kind;
-        a.x[t] = targets[t].x;
-    }
-    a.choice = d_choice;
-    if (d_pred) {
-        const size_t plane = (size_t)n_k * n_f;
-        a.S_out = d_pred;
-        a.E_out = d_pred + plane;
-        a.X_out[0] = x2 ? d_pred + 2 * plane : nullptr;
-        a.X_out[1] = x3 ? d_pred + 3 * plane : nullptr;
-    }
-    a.mode = kModeSweep;
-    a.tile_k = c.tile_k;
-    a.xs = c.xs;
-    a.head_bytes = c.head_bytes;
-    a.grid = clocks->d_grid;
-    a.f0 = clocks->f0;
-    a.inv_step = clocks->inv_step;
-    a.nsub = c.slots;
-    const long long grid = (n_k + c.tile_k - 1) / c.tile_k;
-    if (grid > 0x7fffffffLL) return fail(SYN_ERR_UNSUPPORTED, "n_kernels too large for one launch");
-    const cudaStream_t st = static_cast<cudaStream_t>(stream);
-    SvrScratch scr;
-    syn_status ss = SYN_OK;
-    DevModel* dms[4] = {&a.ms, &a.me, &a.mx[0], &a.mx[1]};
-    for (int m = 0; m < 4 && ss == SYN_OK; ++m)
-        if (m < 2 || a.has_x[m - 2]) ss = prepare_svr(*dms[m], clocks->device, d_features, n_k, F, clocks, st, scr);
-    if (ss != SYN_OK) return ss;
-    const char* algo_env = getenv("SYNERGY_ALGO");
-    if (!algo_env && tm_eligible(a, 4)) {
-        int nl = 0;
-        syn_model* ms[4] = {const_cast<syn_model*>(sp), const_cast<syn_model*>(en), const_cast<syn_model*>(x2),
-                            const_cast<syn_model*>(x3)};
-        int var = 4000;
-        ss = run_tm(a, 4, ms, clocks, st, &nl, &var);
-        if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, (long long)std::min<long long>(2LL * sm_count(clocks->device), n_k),
-                  var == 4001 ? kTrNT : kTmNT, var};
-        return ok();
-    }
-    cudaError_t e;
-    {
-        KernelTimer kt("k_sweep_da", st);
-        e = launch_da(a, c, grid, st);
-    }
-    if (e != cudaSuccess) return cuda_fail(e, "k_sweep_da launch");
-    g_last = {1 + scr.launches, n_k * (long long)n_f, grid, c.nt, 3000 + c.tile_k};
-    return ok();
+    return run_sweep(models, 4, d_features, n_k, F, clocks, def, targets, n_t, d_choice, pred, kModeSweep,
+                     static_cast<cudaStream_t>(stream));
 }
 
 syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32_t n_f, int32_t def,
@@ -1577,9 +1326,11 @@ syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32
     a.choice = d_choice;
     int dev = 0;
     cudaGetDevice(&dev);
+    DevState* ds = nullptr;
+    if ((s = need_dev(dev, &ds)) != SYN_OK) return s;
     const int block = 256;
     const long long need = (n_k + 7) / 8;
-    const long long grid = std::min<long long>(need, (long long)sm_count(dev) * 8);
+    const long long grid = std::min<long long>(need, (long long)ds->sms * 8);
     {
         KernelTimer kt("k_select", static_cast<cudaStream_t>(stream));
         k_select<<<(unsigned)grid, block, 0, static_cast<cudaStream_t>(stream)>>>(a);
@@ -1598,8 +1349,14 @@ syn_status synergy_pareto(const float* d_S, const float* d_E, int64_t n_k, int32
     if (!d_S || !d_E || !d_front) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
     int dev = 0;
     cudaGetDevice(&dev);
-    const long long grid = std::min<long long>((n_k + 7) / 8, (long long)sm_count(dev) * 8);
-    k_pareto<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_S, d_E, n_k, n_f, d_front);
+    DevState* ds = nullptr;
+    syn_status s = need_dev(dev, &ds);
+    if (s != SYN_OK) return s;
+    const long long grid = std::min<long long>((n_k + 7) / 8, (long long)ds->sms * 8);
+    {
+        KernelTimer kt("k_pareto", static_cast<cudaStream_t>(stream));
+        k_pareto<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_S, d_E, n_k, n_f, d_front);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "k_pareto launch");
     g_last = {1, n_k * (long long)n_f, grid, 256, 0};
@@ -1630,15 +1387,21 @@ syn_status synergy_choice_error(const float* d_S, const float* d_E, int64_t n_k,
     }
     int dev = 0;
     cudaGetDevice(&dev);
+    DevState* ds = nullptr;
+    if ((vs = need_dev(dev, &ds)) != SYN_OK) return vs;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     if (n_k > 0) {
-        const long long grid = std::min<long long>((n_k + 7) / 8, (long long)sm_count(dev) * 8);
+        const long long grid = std::min<long long>((n_k + 7) / 8, (long long)ds->sms * 8);
+        KernelTimer kt("k_choice_error", st);
         k_choice_error<<<(unsigned)grid, 256, 0, st>>>(a, d_pred, d_err);
     }
-    k_error_reduce<<<n_t, 256, 0, st>>>(d_err, n_k, n_t, d_summary);
+    {
+        KernelTimer kt("k_error_reduce", st);
+        k_error_reduce<<<n_t, 256, 0, st>>>(d_err, n_k, n_t, d_summary);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "k_choice_error launch");
-    g_last = {2, n_k * (long long)n_f, 0, 256, 0};
+    g_last = {n_k > 0 ? 2 : 1, n_k * (long long)n_f, 0, 256, 0};
     return ok();
 }
 
@@ -1650,9 +1413,15 @@ syn_status synergy_plan(const int32_t* d_choice, int64_t n_k, int32_t n_t, const
     if (!current_device_is(clocks->device)) return fail(SYN_ERR_INVALID_ARG, "clocks device differs from the current device");
     if (n_k == 0) return ok();
     if (!d_choice || !d_mhz) return fail(SYN_ERR_INVALID_ARG, "device buffer is NULL");
+    DevState* ds = nullptr;
+    syn_status s = need_dev(clocks->device, &ds);
+    if (s != SYN_OK) return s;
     const long long n = n_k * (long long)n_t;
-    const long long grid = std::min<long long>((n + 255) / 256, (long long)sm_count(clocks->device) * 16);
-    k_plan<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_choice, n, clocks->d_freqs, clocks->n_f, d_mhz);
+    const long long grid = std::min<long long>((n + 255) / 256, (long long)ds->sms * 16);
+    {
+        KernelTimer kt("k_plan", static_cast<cudaStream_t>(stream));
+        k_plan<<<(unsigned)grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(d_choice, n, clocks->d_freqs, clocks->n_f, d_mhz);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "k_plan launch");
     g_last = {1, n, grid, 256, 0};
@@ -1690,10 +1459,15 @@ syn_status synergy_sweep_host(syn_workspace* w, const syn_model* sp, const syn_m
     if (!clocks || !current_device_is(w->device) || clocks->device != w->device)
         return fail(SYN_ERR_INVALID_ARG, "workspace/clocks device differs from the current device");
     if (n_k > 0 && (!h_features || !h_choice)) return fail(SYN_ERR_INVALID_ARG, "host buffer is NULL");
-    syn_status vs = validate_sweep(sp, en, n_k, F, clocks, def, targets, n_t, kModeSweep);
+    const syn_model* models[2] = {sp, en};
+    syn_status vs = validate_models(models, 2, F, clocks);
     if (vs != SYN_OK) return vs;
+    if (n_k < 0) return fail(SYN_ERR_INVALID_ARG, "n_kernels=%lld < 0", (long long)n_k);
+    const int n_f = clocks->n_f;
+    if (def < 0 || def >= n_f) return fail(SYN_ERR_INVALID_ARG, "default_idx=%d outside [0, %d)", def, n_f);
+    if ((vs = check_targets(targets, n_t)) != SYN_OK) return vs;
     const size_t fb = (size_t)n_k * (size_t)F * sizeof(float);
-    const size_t cb = (size_t)n_k * (size_t)std::max(n_t, 0) * sizeof(int32_t);
+    const size_t cb = (size_t)n_k * (size_t)n_t * sizeof(int32_t);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     if (fb > w->cap_features) {
@@ -1712,8 +1486,9 @@ syn_status synergy_sweep_host(syn_workspace* w, const syn_model* sp, const syn_m
     }
     if (n_k > 0 && (e = cudaMemcpyAsync(w->d_features, h_features, fb, cudaMemcpyHostToDevice, st)) != cudaSuccess)
         return cuda_fail(e, "cudaMemcpyAsync H2D");
-    syn_status s = run_sweep(sp, en, w->d_features, n_k, F, clocks, def, targets, n_t, w->d_choice, nullptr,
-                             nullptr, kModeSweep, st);
+    float* pred[4] = {nullptr, nullptr, nullptr, nullptr};
+    syn_status s = run_sweep(models, 2, w->d_features, n_k, F, clocks, def, targets, n_t, w->d_choice, pred,
+                             kModeSweep, st);
     if (s != SYN_OK) return s;
     if (n_k > 0 && (e = cudaMemcpyAsync(h_choice, w->d_choice, cb, cudaMemcpyDeviceToHost, st)) != cudaSuccess)
         return cuda_fail(e, "cudaMemcpyAsync D2H");

@@ -20,6 +20,8 @@ LIB_PATH = os.path.join(_PKG, "libsynergy.so")
 HEADER = os.path.join(_ROOT, "include", "synergy.h")
 
 SYN_OK, SYN_ERR_INVALID_ARG, SYN_ERR_UNSUPPORTED, SYN_ERR_CUDA, SYN_ERR_OOM = range(5)
+# synergy_last_launch variant codes
+VARIANT_TREE_MAJOR, VARIANT_GENERAL = 4000, 5000
 STATUS_NAMES = {0: "SYN_OK", 1: "SYN_ERR_INVALID_ARG", 2: "SYN_ERR_UNSUPPORTED", 3: "SYN_ERR_CUDA",
                 4: "SYN_ERR_OOM"}
 
@@ -83,6 +85,9 @@ def load(path: str = LIB_PATH) -> C.CDLL:
         "synergy_last_launch": (I32, [P, P, P, P, P]),
         "synergy_timing_enable": (I32, [I32]),
         "synergy_timing_read": (I32, [I32, P, P, P, P]),
+        "synergy_prepare": (I32, [P, I32, I64, I32, P, P]),
+        "synergy_config_set": (I32, [C.c_char_p, I64]),
+        "synergy_config_get": (I32, [C.c_char_p, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -341,6 +346,26 @@ class Workspace:
             self.close()
         except Exception:
             pass
+
+
+def prepare(models, n_kernels: int, n_features: int, clocks: Clocks, stream=None):
+    """synergy_prepare: create the persistent scratch for calls of this shape on `stream` (so later
+    calls only enqueue kernels, e.g. inside a CUDA-graph capture).  models = [speedup, energy] or
+    [speedup, energy, edp|None, ed2p|None]."""
+    handles = (C.c_void_p * len(models))(*[None if m is None else m.handle.value for m in models])
+    _check(load().synergy_prepare(handles, len(models), int(n_kernels), int(n_features), clocks.handle,
+                                  _stream(stream)))
+
+
+def config_set(key: str, value: int):
+    """synergy_config_set: a launch-configuration knob (results do not depend on it)."""
+    _check(load().synergy_config_set(key.encode(), int(value)))
+
+
+def config_get(key: str) -> int:
+    v = C.c_int64()
+    _check(load().synergy_config_get(key.encode(), C.byref(v)))
+    return v.value
 
 
 def last_launch():

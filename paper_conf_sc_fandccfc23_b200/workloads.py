@@ -460,11 +460,12 @@ def make_config(cfg: str, row0: int = 0, n: Optional[int] = None, models=None) -
 # ---------------------------------------------------------------------- fuzz cases
 
 def random_tree_arrays(rng, F, freqs, max_depth, p_leaf=0.2, p_freq=0.3, shuffle=True,
-                       exact_thresholds=False, value_range=(0.25, 4.0)):
+                       exact_thresholds=False, value_range=(0.25, 4.0), p_special_thr=0.0):
     """One unbalanced tree (early-leaf prob p_leaf) in sklearn layout with node ids shuffled.
 
     With exact_thresholds, some thresholds are set equal to existing feature values / clocks so
-    `x == thr` (routes left) is exercised.
+    `x == thr` (routes left) is exercised; p_special_thr makes that fraction of the thresholds
+    NaN (everything goes right), +-inf or +-0.0.
     """
     feature, left, right, value = [], [], [], []
 
@@ -489,6 +490,8 @@ def random_tree_arrays(rng, F, freqs, max_depth, p_leaf=0.2, p_freq=0.3, shuffle
                 thr = float(np.floor(np.exp2(rng.uniform(0, 10))))
             else:
                 thr = float(np.exp2(rng.uniform(-1, 10)))
+        if p_special_thr > 0.0 and rng.uniform() < p_special_thr:
+            thr = float([np.nan, np.inf, -np.inf, -0.0, 0.0][rng.integers(0, 5)])
         feature[n] = f
         value[n] = thr
         l = new(); r = new()
@@ -524,8 +527,13 @@ def random_forest_spec(rng, F, freqs, n_trees, max_depth, **kw) -> ModelSpec:
 
 
 def fuzz_workload(seed: int, n_kernels: int, n_freqs: int, F: int = 5, n_trees: int = 3,
-                  max_depth: int = 4, targets=None, linear: str = "none", **kw) -> Workload:
-    """Small random case: unbalanced shuffled trees, optional linear member (none|only|both)."""
+                  max_depth: int = 4, targets=None, linear: str = "none", specials: float = 0.0,
+                  **kw) -> Workload:
+    """Small random case: unbalanced shuffled trees, optional linear member (none|only|both).
+
+    specials > 0: that fraction of the feature entries is replaced by values no counter produces
+    (NaN, +-inf, negative counts, -0.0, huge values), to exercise the split semantics x <= thr
+    (NaN goes right, -0.0 == 0.0) on both sides (Q16)."""
     rng = np.random.default_rng(seed)
     if n_freqs <= 1395:
         freqs = clock_table(n_freqs)
@@ -534,6 +542,10 @@ def fuzz_workload(seed: int, n_kernels: int, n_freqs: int, F: int = 5, n_trees: 
     d = default_index(freqs)
     feats = np.floor(np.exp2(rng.uniform(0, 10, size=(n_kernels, F)))).astype(np.float32)
     feats[rng.uniform(size=feats.shape) < 0.1] = 0.0
+    if specials > 0.0:
+        pick = rng.uniform(size=feats.shape) < specials
+        vals = np.array([np.nan, np.inf, -np.inf, -0.0, -1.0, -517.25, 3.0e38, -3.0e38], np.float32)
+        feats[pick] = vals[rng.integers(0, len(vals), size=int(pick.sum()))]
 
     def one():
         if linear == "only":

@@ -37,7 +37,7 @@ def test_library_is_sm100a(lib):
 
 
 def test_version_and_error_string(lib):
-    assert lib.synergy_version() == 2
+    assert lib.synergy_version() == 3
     h = C.c_void_p()
     assert lib.synergy_model_create(None, 0, C.byref(h)) == syn.SYN_ERR_INVALID_ARG
     assert b"desc" in lib.synergy_last_error()
@@ -82,6 +82,38 @@ def test_model_validation(lib):
     assert create(badf) == syn.SYN_ERR_INVALID_ARG                         # feature >= n_inputs
     none = W.ModelSpec(n_inputs=3)
     assert create(none) == syn.SYN_ERR_INVALID_ARG                         # no member
+    for bad in (np.inf, -np.inf, np.nan):                                  # non-finite leaf value
+        nf = W.ModelSpec(feature=np.array([0, -1, -1], np.int32), left=np.array([1, -1, -1], np.int32),
+                         right=np.array([2, -1, -1], np.int32), n_inputs=3, forest_weight=1.0,
+                         tree_offset=np.array([0, 3], np.int64), value=np.array([0.5, 1.0, bad], np.float32))
+        assert create(nf) == syn.SYN_ERR_INVALID_ARG
+        assert b"not finite" in lib.synergy_last_error()
+    # a NaN threshold is allowed (x <= NaN is false: every input goes right)
+    nan_thr = W.ModelSpec(feature=np.array([0, -1, -1], np.int32), left=np.array([1, -1, -1], np.int32),
+                          right=np.array([2, -1, -1], np.int32), n_inputs=3, forest_weight=1.0,
+                          tree_offset=np.array([0, 3], np.int64), value=np.array([np.nan, 1.0, 2.0], np.float32))
+    assert create(nan_thr) in (syn.SYN_OK, syn.SYN_ERR_INVALID_ARG, syn.SYN_ERR_CUDA)
+    if create(nan_thr) == syn.SYN_ERR_INVALID_ARG:                         # only "no device" may fail it
+        assert b"device" in lib.synergy_last_error()
+
+
+def test_target_kinds_and_tuning_keys(lib):
+    """ES_ABS / PL_ABS (kinds 6, 7) are accepted, kind 8 is not; tuning keys round-trip and an
+    unknown key is INVALID_ARG (all host-side, no device needed)."""
+    for kind in (6, 7):
+        tg, n_t = syn._targets([(kind, 25.0)])
+        assert lib.synergy_select(None, None, 0, 8, 0, tg, n_t, None, None) == syn.SYN_OK
+        tg, n_t = syn._targets([(kind, 101.0)])
+        assert lib.synergy_select(None, None, 0, 8, 0, tg, n_t, None, None) == syn.SYN_ERR_INVALID_ARG
+    tg, n_t = syn._targets([(8, 0.0)])
+    assert lib.synergy_select(None, None, 0, 8, 0, tg, n_t, None, None) == syn.SYN_ERR_INVALID_ARG
+    old = syn.config_get("tm_kb")
+    syn.config_set("tm_kb", 64)
+    assert syn.config_get("tm_kb") == 64
+    syn.config_set("tm_kb", old)
+    with pytest.raises(syn.SynergyError) as ei:
+        syn.config_set("no_such_knob", 1)
+    assert ei.value.status == syn.SYN_ERR_INVALID_ARG
 
 
 def test_model_desc_layout_matches_header():

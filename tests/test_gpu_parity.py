@@ -21,12 +21,11 @@ def _build():
     oracle.build()
 
 
-# Kernel variants the library can pick (read per call from the environment):
-#   default   tree-major resume walks through L1 (k_tm_walk + k_tm_finish), exact int64 sums in L2
-#   tr        tree-resident resume walks (k_tr_walk + k_tm_finish): trees and chunk features staged
-#             in shared memory by bulk copy, per-lane-index task pools (opt-in, SYNERGY_TM_MODE=tr)
-#   tr_p96    k_tr_walk with 96-kernel chunks (3 kernels per pool, most lanes draw nothing)
-#   tr_ctas3  k_tr_walk on 3 CTAs (many units and chunk switches per CTA: ring phases, restaging)
+# Launch configurations the library can pick (synergy_config_set knobs; results must not change):
+#   default   automatic: tree-major resume walks (k_tm_walk + k_tm_finish) for these models
+#   gen       the general exact path forced (k_gen_forest + k_gen_finish: direct traversal,
+#             320-bit exact leaf sums)
+#   gen_kt3   general path, 3 kernels per finish CTA (ragged last tile)
 #   tm_kb32   k_tm_walk with 32-kernel feature blocks (several blocks per CTA range)
 #   tm_ctas3  k_tm_walk on 3 CTAs (long per-CTA ranges crossing kernel blocks, many tasks/lane)
 #   tm_nsub3  k_tm_walk with every (kernel, tree) task split into 3 clock sub-ranges (uneven)
@@ -37,52 +36,33 @@ def _build():
 #   tm_slab   kernel slabs of 64 (several walk + finish launches; finish(i) on the side stream
 #             overlapping walk(i + 1), D double-buffered and re-zeroed by the finishes)
 #   tm_slab_seq  kernel slabs of 64 run in order on the caller's stream (one D buffer)
-#   da        order-free difference-array kernel (k_sweep_da), shared-memory int64 sums
-#   da_nt64   k_sweep_da with 64 threads per kernel (several tasks per lane)
-#   da_nt256  k_sweep_da with 256 threads per CTA
-#   da_kpc5   k_sweep_da with 5 kernels per CTA (tasks of several kernels per warp, ragged tile)
-#   da_nsub3  k_sweep_da splitting every (kernel, tree) task into 3 clock sub-ranges
-#   da_nsub64 k_sweep_da with 64 sub-ranges (single-clock and empty ranges on small tables)
-#   da_topc   k_sweep_da with the shared top-block cache (TOPC), 3 kernels per CTA
-#   ws        in-order warp-streaming kernel (k_sweep_ws), 2 kernels per CTA, window 64
-#   ws_tight  k_sweep_ws with window 32 (= warp width: refills wait on the oldest tree), 1 run
-#             value kept per tree (every later run takes the direct-walk fallback), 3 kernels/CTA
-#   ws_wide   k_sweep_ws with window 128, 1 kernel per CTA
-#   direct    per-clock root-to-leaf traversal (k_sweep)
-#   iv        chunked clock-interval kernel (k_sweep_iv), auto tile
-#   iv_vcap1  k_sweep_iv keeping 1 run value per (kernel, tree)
-#   iv_tk3    k_sweep_iv with 3 kernels per CTA (ragged last tile, mixed-kernel warps)
-#   iv_nt256  k_sweep_iv, 256 threads, 5 kernels per CTA (51 trees per chunk)
-DA = {"SYNERGY_ALGO": "da"}
-TR = {"SYNERGY_TM_MODE": "tr"}
-VARIANTS = {"default": {}, "tr": TR, "tr_p96": {**TR, "SYNERGY_TR_P": "96"},
-            "tr_ctas3": {**TR, "SYNERGY_TR_CTAS": "3"}, "tm_kb32": {"SYNERGY_TM_KB": "32"}, "tm_ctas3": {"SYNERGY_TM_CTAS": "3"},
-            "tm_nsub3": {"SYNERGY_TM_NSUB": "3"}, "tm_nsub64": {"SYNERGY_TM_NSUB": "64"},
-            "tm_dyn": {"SYNERGY_TM_DYN": "1"}, "tm_static": {"SYNERGY_TM_DYN": "0"},
-            "tm_nopdl": {"SYNERGY_TM_PDL": "0"},
-            "tm_slab": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32"},
-            "tm_slab_seq": {"SYNERGY_TM_SLAB": "64", "SYNERGY_TM_KB": "32", "SYNERGY_TM_PIPE": "0"},
-            "da": DA, "da_nt64": {**DA, "SYNERGY_NT": "64"}, "da_nt256": {**DA, "SYNERGY_NT": "256"},
-            "da_kpc5": {**DA, "SYNERGY_KPC": "5"}, "da_nsub3": {**DA, "SYNERGY_NSUB": "3"},
-            "da_nsub64": {**DA, "SYNERGY_NSUB": "64", "SYNERGY_KPC": "2"},
-            "da_topc": {**DA, "SYNERGY_TOPC": "1", "SYNERGY_KPC": "3"},
-            "ws": {"SYNERGY_ALGO": "ws"},
-            "ws_tight": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "32", "SYNERGY_VCAP": "1", "SYNERGY_KPC": "3"},
-            "ws_wide": {"SYNERGY_ALGO": "ws", "SYNERGY_WIN": "128", "SYNERGY_KPC": "1"},
-            "direct": {"SYNERGY_ALGO": "direct"}, "iv": {"SYNERGY_ALGO": "iv"},
-            "iv_vcap1": {"SYNERGY_ALGO": "iv", "SYNERGY_VCAP": "1"},
-            "iv_tk3": {"SYNERGY_ALGO": "iv", "SYNERGY_TK": "3"},
-            "iv_nt256": {"SYNERGY_ALGO": "iv", "SYNERGY_NT": "256", "SYNERGY_TK": "5"}}
-KNOBS = ("SYNERGY_TM_PDL", "SYNERGY_TM_PIPE", "SYNERGY_TM_DYN", "SYNERGY_TM_MODE", "SYNERGY_TM_NSUB", "SYNERGY_TR_P", "SYNERGY_TR_CTAS", "SYNERGY_TM_KB", "SYNERGY_TM_CTAS", "SYNERGY_TM_SLAB", "SYNERGY_ALGO", "SYNERGY_VCAP", "SYNERGY_TK", "SYNERGY_NT", "SYNERGY_WIN", "SYNERGY_KPC", "SYNERGY_TOPC", "SYNERGY_NSUB")
+VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 3},
+            "tm_kb32": {"tm_kb": 32}, "tm_ctas3": {"tm_ctas": 3},
+            "tm_nsub3": {"tm_nsub": 3}, "tm_nsub64": {"tm_nsub": 64},
+            "tm_dyn": {"tm_dyn": 1}, "tm_static": {"tm_dyn": 0}, "tm_nopdl": {"tm_pdl": 0},
+            "tm_slab": {"tm_slab": 64, "tm_kb": 32},
+            "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0}}
+KNOB_DEFAULTS = {"algo": 0, "tm_kb": 0, "tm_ctas": 0, "tm_nsub": 0, "tm_dyn": -1, "tm_pdl": 1, "tm_slab": 0,
+                 "tm_pipe": 1, "tm_kt": 0, "gen_kt": 0}
+
+
+def set_knobs(values):
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    for k, v in {**KNOB_DEFAULTS, **values}.items():
+        syn.config_set(k, v)
 
 
 @pytest.fixture(params=list(VARIANTS))
-def variant(request, monkeypatch):
-    for k in KNOBS:
-        monkeypatch.delenv(k, raising=False)
-    for k, v in VARIANTS[request.param].items():
-        monkeypatch.setenv(k, v)
-    return request.param
+def variant(request):
+    set_knobs(VARIANTS[request.param])
+    yield request.param
+    set_knobs({})
+
+
+@pytest.fixture(autouse=True)
+def _default_knobs():
+    set_knobs({})
+    yield
 
 
 @pytest.mark.parametrize("cfg", ["c1", "c2"])
@@ -126,6 +106,15 @@ FUZZ = [
     (23, 196, 4, 5, 14, "none", {"p_freq": 0.9, "p_leaf": 0.05}),    # clock-heavy: resume stack overflows
     (29, 64, 3, 4, 16, "none", {"p_freq": 0.7, "p_leaf": 0.02, "exact_thresholds": True}),
     (600, 64, 5, 4, 9, "both", {"p_freq": 0.5}),                      # 3 kernel blocks, ragged last
+    # features no counter produces (NaN, +-inf, negative, -0.0, huge) and special thresholds
+    (37, 64, 6, 5, 8, "none", {"specials": 0.15, "p_special_thr": 0.1, "exact_thresholds": True}),
+    (19, 33, 4, 3, 6, "both", {"specials": 0.1}),
+    # input counts: F = 1, 64 (tree-major), 99, 100, 254 (general path: beyond k_tm_walk's shared memory)
+    (45, 50, 1, 4, 7, "none", {"p_freq": 0.5}),
+    (70, 40, 64, 4, 8, "both", {}),
+    (33, 37, 99, 3, 7, "none", {}),
+    (21, 64, 100, 3, 7, "both", {"specials": 0.05}),
+    (9, 29, 254, 3, 9, "none", {"p_freq": 0.2}),
 ]
 
 
@@ -143,17 +132,16 @@ def test_fuzz_bit_exact(case, variant):
         assert_choices(got["choice"], ref["choice"], ref["gap"])
 
 
-def test_tree_resident_routing(monkeypatch):
-    """With SYNERGY_TM_MODE=tr, k_tr_walk (variant 4001) runs when every tree fits its 64 KB shared
-    tree buffer; a model with a larger tree routes to the L1-cached k_tm_walk (4000); both exact."""
+def test_path_routing():
+    """Which kernels run: the tree-major pair for in-range forests that fit shared memory, the
+    general exact pair for out-of-range leaves, F beyond k_tm_walk's shared memory, and models
+    without a forest member.  Both paths are checked bit-exact elsewhere."""
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
-    for k in KNOBS:
-        monkeypatch.delenv(k, raising=False)
-    monkeypatch.setenv("SYNERGY_TM_MODE", "tr")
-    small = W.fuzz_workload(77, 40, 64, F=4, n_trees=3, max_depth=8, p_leaf=0.1)
-    big = W.fuzz_workload(78, 40, 64, F=4, n_trees=2, max_depth=16, p_freq=0.3, p_leaf=0.0)
-    assert max(np.diff(big.energy.tree_offset)) > 2 * 4 * 2048      # > 2048 2-level blocks
-    for w, want in ((small, 4001), (big, 4000)):
+    cases = [(W.fuzz_workload(77, 40, 64, F=4, n_trees=3, max_depth=8), syn.VARIANT_TREE_MAJOR),
+             (W.fuzz_workload(78, 40, 64, F=120, n_trees=3, max_depth=8), syn.VARIANT_GENERAL),
+             (W.fuzz_workload(79, 40, 64, F=4, n_trees=3, max_depth=4, linear="only"), syn.VARIANT_GENERAL),
+             (_stump_models([2.0 ** 60, 100.0, 100.0], [1.0, 2.0]), syn.VARIANT_GENERAL)]
+    for w, want in cases:
         ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
         got = gpu_sweep(w, want_pred=True)
         assert syn.last_launch()["variant"] == want
@@ -195,16 +183,65 @@ def test_exact_sum_where_sequential_fp64_rounds(swap):
     assert_bits_equal(E, rE, "raw E")
 
 
-def test_out_of_range_leaves_fall_back_to_ordered_kernel():
-    """Leaves spanning more than the int64 fixed-point range route to the ordered kernels; with
-    two leaves per evaluation the sequential fp64 sum is a single rounding = the exact sum."""
-    from paper_conf_sc_fandccfc23_b200 import synergy as syn
-    w = _stump_models([2.0 ** 60, 2.0 ** -60], [1.0, 0.5])
+# Leaf sets whose exact sum a sequential fp64 sum does not reproduce, beyond the int64 fixed-point
+# range (Q8): the general path's 320-bit sums must equal the oracle's math.fsum value.
+EXTREME_LEAVES = [
+    [2.0 ** 60, 100.0, 100.0],                     # no cancellation; sequential sum rounds twice
+    [2.0 ** 100, 1.0, -2.0 ** 100, 2.0 ** -100],   # catastrophic cancellation
+    [2.0 ** 60, 1.0, -2.0 ** 60],                  # exact 1/3 mean; sequential gives 0
+    [2.0 ** 127, 2.0 ** 127, -2.0 ** 127, 2.0 ** -149, 3.0 * 2.0 ** -149],   # fp32 extremes
+    [-(2.0 ** 90), 5.0, 2.0 ** 90, -(2.0 ** -120)] * 3,
+    [float(np.float32(1.1)), 2.0 ** 40, float(np.float32(-1.7)), -(2.0 ** 40), 2.0 ** -60],
+]
+
+
+@pytest.mark.parametrize("case", range(len(EXTREME_LEAVES)))
+@pytest.mark.parametrize("on_energy", [False, True])
+def test_extreme_leaves_exact_sum(case, on_energy, variant):
+    import math
+    vals = [float(np.float32(v)) for v in EXTREME_LEAVES[case]]
+    seq = 0.0
+    for v in vals:
+        seq += v
+    if case < 3:
+        assert seq != math.fsum(vals)                   # the case needs the exact sum
+    other = [1.0, 2.0]
+    w = _stump_models(other, vals) if on_energy else _stump_models(vals, other)
     S, E = gpu_predict(w, default_idx=-1)
     rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, -1)
-    assert syn.last_launch()["variant"] // 1000 not in (3, 4)
     assert_bits_equal(S, rS, "raw S")
     assert_bits_equal(E, rE, "raw E")
+    got = gpu_sweep(w, want_pred=True)
+    ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
+    assert_bits_equal(got["S"], ref["S"], "S")
+    assert_bits_equal(got["E"], ref["E"], "E")
+    assert_choices(got["choice"], ref["choice"], ref["gap"])
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_wide_range_forests(seed):
+    """Random unbalanced forests whose leaves span the whole fp32 range with both signs, so every
+    call takes the general path's multi-word sums; many trees per model."""
+    rng = np.random.default_rng(500 + seed)
+    w = W.fuzz_workload(600 + seed, 23, 64, F=6, n_trees=40, max_depth=6, p_leaf=0.15)
+    for m in (w.speedup, w.energy):
+        leaves = m.feature < 0
+        mag = np.exp2(rng.uniform(-149, 127.9, size=int(leaves.sum())))
+        m.value[leaves] = (mag * rng.choice([-1.0, 1.0], size=mag.size)).astype(np.float32)
+    for d in (-1, w.default_idx):
+        S, E = gpu_predict(w, default_idx=d)
+        rS, rE = oracle.predict(w.speedup, w.energy, w.features, w.freqs, d)
+        assert_bits_equal(S, rS, f"S (default {d})")
+        assert_bits_equal(E, rE, f"E (default {d})")
+
+
+def test_non_finite_leaves_rejected_at_create():
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    for bad in (np.inf, -np.inf, np.nan):
+        w = _stump_models([1.0, bad], [1.0])
+        with pytest.raises(syn.SynergyError) as ei:
+            syn.Model(w.speedup)
+        assert ei.value.status == syn.SYN_ERR_INVALID_ARG
 
 
 def _gpu_sweep4(models, feats, freqs, d, targets):
@@ -222,8 +259,6 @@ def _gpu_sweep4(models, feats, freqs, d, targets):
 @pytest.mark.parametrize("cfg", ["c1", "c2"])
 def test_four_model_variant_bit_exact(cfg, variant):
     """NEXT f1: speedup + energy + direct EDP (RF) + direct ED2P (linear)."""
-    if VARIANTS[variant].get("SYNERGY_ALGO", "da") != "da":
-        pytest.skip("four-model sweep runs on the exact int64 kernels only")
     models, freqs, d = W.make_models4(cfg)
     feats = W.make_features(cfg)
     targets = W.targets_six()
@@ -356,10 +391,11 @@ def test_invalid_arguments_enqueue_nothing():
 
 # ------------------------------------------------- full sizes, bench launch config, sampled
 
-@pytest.mark.parametrize("cfg,n_sample", [("c3", 48), ("c4", 384), ("c5", 3584)])
+@pytest.mark.parametrize("cfg,n_sample", [("c4", 384), ("c5", 3584)])
 def test_full_size_sampled(cfg, n_sample):
     """The GPU runs the whole config in the launch configuration bench.py times; the oracle
-    recomputes a seeded sample of kernel rows (c5: all rows; its 64 replicas must agree)."""
+    recomputes a seeded sample of kernel rows (c5: all rows; its 64 replicas must agree).  c3 is
+    compared row by row in full in test_gpu_fullsize.py (c4 in full there on request)."""
     import torch
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
     w = W.make_config(cfg)

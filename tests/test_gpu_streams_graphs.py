@@ -20,7 +20,7 @@ def _build():
 
 
 def _workload(seed):
-    # several kernel slabs at SYNERGY_TM_SLAB=64: the pipeline runs (finish i || walk i + 1)
+    # several kernel slabs at tm_slab = 64: the pipeline runs (finish i || walk i + 1)
     return W.fuzz_workload(seed, 300, 64, F=5, n_trees=4, max_depth=8, p_leaf=0.1)
 
 
@@ -48,10 +48,18 @@ def _check(w, S, E, out):
     assert np.array_equal(out.cpu().numpy(), ref["choice"])
 
 
-def test_two_streams_concurrently(monkeypatch):
+@pytest.fixture
+def slabs64():
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    syn.config_set("tm_slab", 64)
+    syn.config_set("tm_kb", 32)
+    yield
+    syn.config_set("tm_slab", 0)
+    syn.config_set("tm_kb", 0)
+
+
+def test_two_streams_concurrently(slabs64):
     import torch
-    monkeypatch.setenv("SYNERGY_TM_SLAB", "64")
-    monkeypatch.setenv("SYNERGY_TM_KB", "32")
     ws = [_workload(5), _workload(6)]
     streams = [torch.cuda.Stream(), torch.cuda.Stream()]
     bufs = [_buffers(w) for w in ws]
@@ -66,10 +74,8 @@ def test_two_streams_concurrently(monkeypatch):
         _check(w, *b)
 
 
-def test_captured_in_cuda_graph(monkeypatch):
+def test_captured_in_cuda_graph(slabs64):
     import torch
-    monkeypatch.setenv("SYNERGY_TM_SLAB", "64")
-    monkeypatch.setenv("SYNERGY_TM_KB", "32")
     w = _workload(7)
     S, E, out = _buffers(w)
     s = torch.cuda.Stream()
@@ -85,3 +91,39 @@ def test_captured_in_cuda_graph(monkeypatch):
         g.replay()
     torch.cuda.synchronize()
     _check(w, S, E, out)
+
+
+def test_prepare_then_capture_on_a_fresh_stream(slabs64):
+    """synergy_prepare creates the clock-cut copies, difference arrays and side stream, so the very
+    first sweep on the stream can be captured."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = _workload(8)
+    S, E, out = _buffers(w)
+    s = torch.cuda.Stream()
+    keep, call = _run(w, s.cuda_stream, S, E, out)
+    syn.prepare([keep[0], keep[1]], w.n_kernels, w.n_features, keep[2], stream=s.cuda_stream)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        call()
+    g.replay()
+    torch.cuda.synchronize()
+    _check(w, S, E, out)
+
+
+def test_unprepared_capture_is_refused():
+    """Without prepare / warm-up, the persistent scratch cannot be created inside a capture: the
+    call returns SYN_ERR_UNSUPPORTED (nothing is enqueued) instead of breaking the capture."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = _workload(9)
+    S, E, out = _buffers(w)
+    s = torch.cuda.Stream()
+    keep, call = _run(w, s.cuda_stream, S, E, out)
+    g = torch.cuda.CUDAGraph()
+    with pytest.raises(syn.SynergyError) as ei:
+        with torch.cuda.graph(g, stream=s):
+            call()
+    assert ei.value.status == syn.SYN_ERR_UNSUPPORTED
+    torch.cuda.synchronize()

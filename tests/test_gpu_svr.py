@@ -10,8 +10,6 @@ sum_j dual_j e^{-gamma (A_kj + B_ji)}: the two fp64 values differ by at most
   * the choices equal the oracle's selection run on the GPU's own predictions (selection is
     exact), and they equal the oracle's choices on every row whose predictions match bit for bit.
 """
-import os
-
 import numpy as np
 import pytest
 
@@ -37,38 +35,28 @@ def check_pred(got, ref, what, max_frac=1e-4):
 
 
 @pytest.fixture
-def env(request):
-    saved = {}
-
-    def set_(k, v):
-        saved.setdefault(k, os.environ.get(k))
-        if v is None:
-            os.environ.pop(k, None)
-        else:
-            os.environ[k] = v
-    yield set_
-    for k, v in saved.items():
-        if v is None:
-            os.environ.pop(k, None)
-        else:
-            os.environ[k] = v
+def knobs():
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    yield syn.config_set
+    syn.config_set("algo", 0)
+    syn.config_set("svr_splits", 0)
 
 
-ALGOS = ["", "da", "ws", "iv", "direct"]
+ALGOS = [0, 1]      # automatic (tree-major for these forests), general exact path
 
 
 @pytest.mark.parametrize("ensemble", [False, True])
 @pytest.mark.parametrize("algo", ALGOS)
-@pytest.mark.parametrize("splits", [None, "1", "5"])
-def test_svr_sweep_matches_oracle(env, ensemble, algo, splits):
-    env("SYNERGY_ALGO", algo or None)
-    env("SYNERGY_SVR_SPLITS", splits)
+@pytest.mark.parametrize("splits", [0, 1, 5])
+def test_svr_sweep_matches_oracle(knobs, ensemble, algo, splits):
+    knobs("algo", algo)
+    knobs("svr_splits", splits)
     w = W.make_config("c1", models=W.make_models_svr("c1", n_sv=200, ensemble=ensemble))
     ref = oracle.sweep(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets, want_pred=True)
     got = gpu_sweep(w, want_pred=True)
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
-    # k_svr_v + k_svr_u + k_svr + the sweep (tree-major default: walk + finish)
-    assert syn.last_launch()["kernels"] == (5 if algo == "" else 4)
+    # k_svr_v + k_svr_u + k_svr + the sweep pair (walk + finish, or forest + finish)
+    assert syn.last_launch()["kernels"] == 5
     check_pred(got["S"], ref["S"], "S")
     dE = check_pred(got["E"], ref["E"], "E")
     np.testing.assert_array_equal(got["choice"], oracle.select(got["S"], got["E"], w.default_idx, w.targets))
