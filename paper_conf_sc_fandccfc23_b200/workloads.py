@@ -564,5 +564,6 @@ def fuzz_workload(seed: int, n_kernels: int, n_freqs: int, F: int = 5, n_trees: 
     sp, en = one(), one()
     if targets is None:
         targets = targets_six() + [(ES, 0.0), (ES, 25.0), (ES, 75.0), (ES, 100.0),
-                                   (PL, 0.0), (PL, 25.0), (PL, 75.0), (PL, 100.0)]
+                                   (PL, 0.0), (PL, 25.0), (PL, 75.0), (PL, 100.0),
+                                   (ES_ABS, 40.0), (PL_ABS, 20.0)]
     return Workload(f"fuzz{seed}", feats, freqs, d, sp, en, targets, n_kernels_total=n_kernels)

@@ -122,7 +122,7 @@ FUZZ = [
 def test_fuzz_bit_exact(case, variant):
     n_k, n_f, F, T, D, lin, kw = FUZZ[case]
     w = W.fuzz_workload(1000 + case, n_k, n_f, F=F, n_trees=T, max_depth=D, linear=lin, **kw)
-    targets_a, targets_b = w.targets[:8], w.targets[8:]
+    targets_a, targets_b = w.targets[:9], w.targets[9:]           # <= 16 targets per call
     for tg in (targets_a, targets_b):
         w.targets = tg
         ref = oracle.sweep_workload(w, want_pred=True, with_gap=True)
@@ -351,7 +351,8 @@ def test_standalone_select_on_oracle_predictions_with_invalid_entries():
         E[rng.uniform(size=E.shape) < 0.05] = np.nan
         S[rng.uniform(size=S.shape) < 0.02] = np.inf
         d = int(rng.integers(0, n_f))
-        targets = W.targets_six() + [(W.ES, 100.0), (W.PL, 0.0), (W.ES, 33.0), (W.PL, 100.0)]
+        targets = W.targets_six() + [(W.ES, 100.0), (W.PL, 0.0), (W.ES, 33.0), (W.PL, 100.0),
+                                     (W.ES_ABS, 25.0), (W.PL_ABS, 75.0), (W.ES_ABS, 0.0), (W.PL_ABS, 100.0)]
         ref = oracle.select(S, E, d, targets)
         got = syn.select(torch.from_numpy(S).cuda(), torch.from_numpy(E).cuda(), d, targets).cpu().numpy()
         assert_choices(got, ref)
