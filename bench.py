@@ -1,17 +1,17 @@
 #!/usr/bin/env python
 """bench.py — SYnergy fused predict+select on B200: kernel x frequency evaluations/s.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--impl ours|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...      (one process per GPU, NCCL)
 
 A step = one pass of the whole hot path over one batch: synergy_sweep (model inference for
 every (kernel, clock) pair, default-clock normalisation, per-target objectives, masked argmin;
 PAPER §6.2) on the rank's kernels, then (N > 1) the NCCL all-gather that assembles
-the choice table.  Default workload = BASELINE.json configs[1] (c2: 1000 kernels x 196 clocks,
-100-tree depth-12 forests for speedup and energy, 6 targets) per rank, weak scaling (rank r
-sweeps its own 1000 kernels of the seeded population).  Inputs are resident in HBM; L2 is
-flushed (512 MiB write) between timed steps because the 13 MB model would otherwise stay in L2.
-Prints ONE JSON line on rank 0.
+the choice table.  Default workload = BASELINE.json configs[2] (c3: 100 000 kernels x 196 clocks,
+500-tree depth-12 forests for speedup and energy, ES/PL targets at 25/50/75 %), the largest
+configuration that fits one GPU, per rank, weak scaling (rank r sweeps its own 100 000 kernels of
+the seeded population).  Inputs are resident in HBM; L2 is flushed (512 MiB write) between timed
+steps (the 65 MB models would otherwise stay in L2).  Prints ONE JSON line on rank 0.
 """
 from __future__ import annotations
 
@@ -35,7 +35,7 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=50)
     p.add_argument("--warmup", type=int, default=10)
-    p.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"])
+    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -91,16 +91,27 @@ def load_peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
-def ncu_traffic(cfg, kernel="k_sweep_da"):
+def ncu_traffic(cfg, kernel="k_tm_walk"):
     """dram__bytes_read.sum + dram__bytes_write.sum per launch of `kernel` on `cfg`, from one
     committed ncu --set full capture (profiles/ncu_traffic.json), or None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(path) as f:
             d = json.load(f).get(cfg, {})
-        return d.get(f"{kernel}_dram_bytes_per_launch", d.get("k_sweep_dram_bytes_per_launch") if kernel == "k_sweep_da" else None)
+        return d.get(f"{kernel}_dram_bytes_per_launch")
     except Exception:
         return None
+
+
+def config_dict(cfg, which, world, n_local, flush_mib):
+    """The `config` object of the JSON line (identical for our arm and the reference arm)."""
+    from paper_conf_sc_fandccfc23_b200 import workloads as W
+    n_f = W.CONFIGS[cfg][1]
+    sp, en = bench_models(cfg, which)[:2]
+    return {"workload": workload_desc(cfg, which), "n_kernels_per_rank": n_local, "n_freqs": n_f,
+            "targets": 6, "parallelism": f"dp{world} (kernel axis) + NCCL all-gather of choices",
+            "l2": f"flushed between timed steps ({flush_mib} MiB write)",
+            "decisions_per_eval": decisions_per_eval(sp) + decisions_per_eval(en)}
 
 
 # ------------------------------------------------------------------------- clock sampler
@@ -266,9 +277,10 @@ def run_reference(args, rank, world):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": workload_desc(cfg, args.models), "sample_kernels_per_step": sample,
-                       "decisions_per_eval": dec},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": len(jobs), "kind": "oracle", "sample": desc},
+            "config": config_dict(cfg, args.models, world, n_k if args.scaling == "weak" else -(-n_k // world),
+                                  args.flush_mib),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": len(jobs), "kind": "oracle", "sample": desc,
+                             "sample_kernels_per_step": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -293,7 +305,8 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        import datetime
+        dist.init_process_group("nccl", device_id=dev, timeout=datetime.timedelta(seconds=600))
     if rank == 0:
         B.build()
     if world > 1:
@@ -428,7 +441,7 @@ def main():
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     dec = decisions_per_eval(sp_spec) + decisions_per_eval(en_spec)
     # dominant kernel of the step, timed by the library's events on its launch stream
-    algo = max(ktimes, key=lambda k: ktimes[k][0]) if ktimes else "k_sweep_da"
+    algo = max(ktimes, key=lambda k: ktimes[k][0]) if ktimes else "k_tm_walk"
     kern_avg_s = (ktimes[algo][0] / ktimes[algo][1] / 1e3) if ktimes else statistics.mean(kern_ms) / 1e3
     kernel_share = ktimes[algo][0] / ktimed_ms if ktimes else sum(kern_ms) / total_ms
     per_kernel = {k: {"ms_per_launch": v[0] / v[1], "launches": v[1], "share_of_step": v[0] / ktimed_ms}
@@ -438,8 +451,15 @@ def main():
     hbm_ach = hbm_bytes / kern_avg_s / 1e9
     hbm = {"achieved": hbm_ach, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": hbm_ach / peaks["hbm_gbs"],
            "algorithmic_bytes": hbm_bytes, "peak_source": peak_src}
+    # on-chip ceilings measured on this GPU now (tools/peaks.cu): scattered 32-byte L1-resident
+    # loads (the k_tm_walk block fetch), the same from L2, conflict-free shared-memory reads
+    import tools
+    try:
+        onchip = tools.measure_peaks(local)
+    except Exception as exc:                                       # noqa: BLE001
+        onchip = {"error": str(exc)}
     work = None
-    if rank == 0 and algo in ("k_sweep_da", "k_sweep_ws", "k_tm_walk", "k_tr_walk"):
+    if rank == 0 and algo == "k_tm_walk":
         work = run_walk_work(cfg, row0, n_local, which=args.models)
     if algo == "k_svr":
         # fp64 FMA-pipe roofline: 2 * n_k * n_f * n_SV flops per contraction
@@ -453,29 +473,25 @@ def main():
                     "peak_note": f"fp64 FMA pipe 64 FMA/clk/SM x 2 x {sms} SMs x {sm_max:.0f} MHz (derived; "
                                  "tcgen05 has no fp64 kind)",
                     "hbm": hbm, "per_kernel": per_kernel}
-    elif work is not None:
-        # on-chip L1 roofline: each run walk fetches max(1, ceil(depth/2)) 32-byte
-        # 2-level blocks; counted by the oracle from the inputs (runs of clocks sharing a leaf)
+    elif work is not None and "l1_scatter32_bytes_per_s" in onchip:
+        # on-chip L1 roofline: each resume walk fetches 32-byte 2-level blocks;
+        # counted by tools/workcount.c from the inputs; peak = the measured rate of exactly that
+        # access (independent scattered 256-bit loads hitting L1) on this GPU
         per_launch = max(1.0, ktimes[algo][1] / K)             # kernel-slab launches per step
-        resume = algo in ("k_tm_walk", "k_tr_walk")
-        blocks = work["resume_blocks_per_kernel" if resume else "run_blocks_per_kernel"] * (evals_step // n_f) / per_launch
+        blocks = work["resume_blocks_per_kernel"] * (evals_step // n_f) / per_launch
         achieved = 32.0 * blocks / kern_avg_s / 1e9
-        peak = 128.0 * sms * sm_max * 1e6 / 1e9
+        peak = onchip["l1_scatter32_bytes_per_s"] / 1e9
         roofline = {"bound": "l1", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                    "peak_source": "measured (tools/peaks.cu k_scatter32 on this GPU in this run)",
                     "traffic": ncu_traffic(cfg, algo) if args.models == "rf" else None, "kernel": algo,
                     "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
                     "algorithmic_bytes_per_launch": 32.0 * blocks,
-                    "work": {"unit": "32-byte 2-level block fetches of the " +
-                                     ("resume walks (each run restarts where its path leaves the previous run's)"
-                                      if resume else "run walks (each run restarts at the root)"),
+                    "work": {"unit": "32-byte 2-level block fetches of the resume walks (each run restarts "
+                                     "where its path leaves the previous run's)",
                              "per_launch": blocks,
                              "runs_per_kernel_tree": work["runs_per_kernel_tree"], "counted_on": work["sample"]},
-                    "peak_note": f"L1/TEX load path 128 B/clk/SM x {sms} SMs x {sm_max:.0f} MHz (derived; "
-                                 "not in MEASURED_PEAKS.json)",
-                    "l1_request_view": {"achieved_per_s": blocks / kern_avg_s,
-                                        "peak_per_s": sms * sm_max * 1e6,
-                                        "note": "one 256-bit LDG (one 32-B sector, one L1 request) per block fetch; "
-                                                "peak = 1 scattered request per clk per SM"},
+                    "onchip_peaks_measured": onchip,
+                    "nominal_l1_bytes_per_s": 128.0 * sms * sm_max * 1e6,
                     "decisions_per_s_vs_direct": evals_step * dec / kern_avg_s,
                     "hbm": hbm, "per_kernel": per_kernel}
     else:
@@ -484,8 +500,8 @@ def main():
         roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gdecisions/s",
                     "frac": achieved / peak, "traffic": ncu_traffic(cfg, algo) if args.models == "rf" else None,
                     "kernel": algo, "kernel_ms": kern_avg_s * 1e3, "kernel_share_of_step": kernel_share,
-                    "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision",
-                    "hbm": hbm, "per_kernel": per_kernel}
+                    "peak_note": f"{sms} SMs x {sm_max:.0f} MHz x 32 lanes / 2 L1 wavefronts per decision (derived)",
+                    "onchip_peaks_measured": onchip, "hbm": hbm, "per_kernel": per_kernel}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -499,11 +515,7 @@ def main():
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": K,
                 "warmup": args.warmup, "ms_per_step": total_ms_max / K, "higher_is_better": True,
                 "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": workload_desc(cfg, args.models), "n_kernels_per_rank": n_local,
-                           "n_freqs": n_f, "targets": n_t,
-                           "parallelism": f"dp{world} (kernel axis) + NCCL all-gather of choices",
-                           "l2": f"flushed between timed steps ({args.flush_mib} MiB write)",
-                           "decisions_per_eval": dec},
+                "config": config_dict(cfg, args.models, world, n_local, args.flush_mib),
                 "gpu_launches": launches, "roofline": roofline, "e2e": e2e, "cpu_baseline": cpu,
                 "clocks": clocks}
         print(json.dumps(line), flush=True)
