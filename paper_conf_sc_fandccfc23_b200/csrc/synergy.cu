@@ -208,7 +208,9 @@ const Knobs& knobs() {
 struct DevState {
     std::once_flag once;
     int sms = 148;
-    int optin = 227 * 1024;               // max dynamic shared memory per CTA (opt-in)
+    int optin = 227 * 1024;               // max shared memory per CTA (opt-in)
+    int walk_dyn_max = 0;                 // dynamic shared memory k_tm_walk / k_tm_finish may take
+    int finish_dyn_max = 0;
     cudaError_t init_err = cudaSuccess;
     cudaMemPool_t pool = nullptr;         // library-owned stream-ordered pool (release threshold max)
     std::mutex occ_mu;
@@ -216,9 +218,14 @@ struct DevState {
 };
 DevState g_dev[kMaxDevices];
 
+// Opt a kernel in to the largest dynamic shared memory the device allows next to its static
+// shared memory.
 template <typename K>
-cudaError_t allow_smem(K kernel, int bytes) {
-    return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+cudaError_t allow_smem(K kernel, int optin) {
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, kernel);
+    if (e != cudaSuccess) return e;
+    return cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, optin - (int)fa.sharedSizeBytes);
 }
 
 // Once per device (the attribute is per device): query limits, opt every kernel with dynamic
@@ -245,6 +252,11 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_svr<7>, d.optin));
         chk(allow_smem(k_svr<8>, d.optin));
         chk(allow_smem(k_svr_u, d.optin));
+        cudaFuncAttributes fa;
+        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false>));
+        d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
+        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_finish));
+        d.finish_dyn_max = d.optin - (int)fa.sharedSizeBytes;
         cudaMemPoolProps props;
         memset(&props, 0, sizeof props);
         props.allocType = cudaMemAllocationTypePinned;
@@ -460,8 +472,8 @@ bool tm_eligible(const SweepArgs& a, int nm, const DevState* ds) {
         ++nslot;
     }
     if (tt == 0) return false;
-    if (tm_walk_smem(a.F, tt) > (size_t)ds->optin) return false;
-    return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->optin;
+    if (tm_walk_smem(a.F, tt) > (size_t)ds->walk_dyn_max) return false;
+    return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->finish_dyn_max;
 }
 
 int finish_ctas_per_sm(DevState* ds, int fnt, size_t smem) {
@@ -542,7 +554,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     const int fnt = 256;
     auto fsmem_of = [&](int k) { return tm_finish_smem(nm, k, n_f, a.xs, t.nslot); };
     int kt_cap = 1;
-    while (kt_cap < 8 && fsmem_of(kt_cap + 1) <= std::min<size_t>((size_t)ds->optin, 150 * 1024)) ++kt_cap;
+    while (kt_cap < 8 && fsmem_of(kt_cap + 1) <= std::min<size_t>((size_t)ds->finish_dyn_max, 150 * 1024)) ++kt_cap;
     // the smallest tile whose finish grid fits in one wave of resident CTAs (a partial second wave
     // doubles the finish's latency chain: c5 KT 3 -> 7 = 1195 -> 512 CTAs, 46 -> 37 us); when no
     // tile fits, the largest (kt_cap)
@@ -1069,6 +1081,17 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
                     w[3] = leaf_code | (leaf_code << 8) | (leaf_code << 16);
                 } else {
                     uint32_t codes = (uint32_t)d->feature[b + id];
+                    // the grandchild blocks of a block (a "family", allocated consecutively) never
+                    // straddle a 128-byte line: lanes of a warp that leave the same block for
+                    // different grandchildren then share one L1 line (one wavefront)
+                    int fam = 0;
+                    for (int dd = 0; dd < 2; ++dd) {
+                        const int64_t c = dd ? d->right[b + id] : d->left[b + id];
+                        if (is_leaf(c)) continue;
+                        fam += !is_leaf(d->left[b + c]) + !is_leaf(d->right[b + c]);
+                    }
+                    if (fam >= 2 && (int)((blocks.size() >> 1) & 3) + fam > 4)
+                        blocks.resize(((blocks.size() >> 1) + 3) / 4 * 4 * 2, make_uint4(0, 0, 0, 0));
                     for (int dd = 0; dd < 2; ++dd) {
                         const int64_t c = dd ? d->right[b + id] : d->left[b + id];
                         w[1 + dd] = fbits(c);
