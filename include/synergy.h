@@ -38,10 +38,10 @@
  *     CUDA graph.  A call that would have to create persistent scratch while its stream is being
  *     captured returns SYN_ERR_UNSUPPORTED instead.
  *   - Paths: the tree-major kernels (k_tm_walk + k_tm_finish) when every forest's leaves fit the
- *     int64 fixed-point range and the inputs / trees fit shared memory (about F <= 90 and 25 000
- *     trees per call); otherwise the general exact kernels (k_gen_forest + k_gen_finish: direct
- *     traversal, 320-bit exact leaf sums), which accept every valid model and F <= 254.  Both
- *     return the same bits.
+ *     int64 fixed-point range and the per-tree task table fits shared memory (about 25 000 trees
+ *     per call, any F); otherwise the general exact kernels (k_gen_forest + k_gen_finish: direct
+ *     traversal, 320-bit exact leaf sums), which accept every valid model.  Both return the same
+ *     bits.
  *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
  *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
  *   - Handles (models, clock tables, workspaces) are bound to the device they were created

@@ -75,20 +75,24 @@ struct TmArgs {
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
     int nsub;                    // clock sub-ranges per (kernel, tree) task (small batches)
-    int dyn;                     // k_tm_walk: tasks from a shared counter (small batches)
+    int dyn;                     // k_tm_walk: tasks from a shared counter
 };
 
 // One 2-level block step on clock-cut words (A = {thr(n), thr(c0), thr(c1), codes}, grandchild
-// words B): the three candidate inputs are read from the lane's column xcol ([F + 2] rows of
-// stride NT: the kernel's static features, the walked clock in row F, row F + 1 for folded
-// leaves), then decided.  Returns the grandchild word taken; *cb = smallest cut of the block's
-// left-turn clock splits (+inf if none), *leaf = the word is a leaf value.
-template <int NT>
-__device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, const float* xcol, float& cb, bool& leaf) {
+// words B): the three candidate inputs are the kernel's static features (shared-memory column at
+// xb of the block's feature table [F + 2][KB], row stride rs = 4 KB bytes; row F + 1 = 0 serves
+// folded leaves) or, for clock splits (flag bits), the walked clock clk; then decided.  Returns
+// the grandchild word taken; *cb = smallest cut of the block's left-turn clock splits (+inf if
+// none), *leaf = the word is a leaf value.
+__device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, unsigned xb, unsigned rs, float clk,
+                                            float& cb, bool& leaf) {
     const unsigned codes = A.w;
-    const float xn = xcol[(size_t)(codes & 0xffu) * NT];
-    const float x0 = xcol[(size_t)((codes >> 8) & 0xffu) * NT];
-    const float x1 = xcol[(size_t)((codes >> 16) & 0xffu) * NT];
+    const float fn = lds_f(xb + rs * (codes & 0xffu));
+    const float f0 = lds_f(xb + rs * ((codes >> 8) & 0xffu));
+    const float f1 = lds_f(xb + rs * ((codes >> 16) & 0xffu));
+    const float xn = (codes & kClkN) ? clk : fn;
+    const float x0 = (codes & kClkC0) ? clk : f0;
+    const float x1 = (codes & kClkC1) ? clk : f1;
     const bool l0 = xn <= __uint_as_float(A.x);
     const unsigned tcb = l0 ? A.y : A.z;
     const bool l1 = (l0 ? x0 : x1) <= __uint_as_float(tcb);
@@ -100,70 +104,95 @@ __device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, cons
     return l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
 }
 
+// Per-tree task record in shared memory: everything a task start needs in one 16-byte load.
+struct __align__(16) TmTree {
+    int root;            // root block
+    int slot_off;        // D slot offset of the tree's model (slot * n_f)
+    const uint4* blocks; // the model's clock-cut blocks
+};
+
 // FXALL: every forest of the call has int32 fixed-point leaves (no int64 conversion path).
-template <int NT, bool FXALL>
+// SUB: (kernel, tree) tasks are split into clock sub-ranges (t.nsub > 1, tiny batches).
+template <int NT, bool FXALL, bool SUB>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
     extern __shared__ __align__(16) unsigned char smem[];
     asm volatile("griddepcontrol.launch_dependents;");                       // k_tm_finish may launch early
-    const int n_f = a.n_f, F = a.F, KB = t.kb;
-    int* stk_b = reinterpret_cast<int*>(smem);                               // [kTmS][NT] record blocks
-    float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
-    float* xs = stk_c + kTmS * NT;                                           // [F + 2][NT] lane columns
-    int2* stree = reinterpret_cast<int2*>(xs + (size_t)(F + 2) * NT);       // [TT] {root block, model}
-    __shared__ int s_next;                                                   // dynamic mode: next task offset
-    __shared__ const uint4* s_blocks[4];                                     // per model: clock-cut blocks,
-    __shared__ int s_slot[4], s_fx[4];                                       // D slot offset, int32 leaves,
-    __shared__ double s_scale[4];                                            // fixed-point scale
-    const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
-    constexpr unsigned kEnt = 4u * NT;                                       // bytes between stack entries
-    float* const xcol = xs + threadIdx.x;
-    const unsigned xclk_a = su32(xcol + (size_t)F * NT);
-    xcol[(size_t)(F + 1) * NT] = 0.0f;   // folded-leaf row: either outcome reaches the same leaf
-
+    const int n_f = a.n_f, F = a.F, KB = t.kb, KBL = t.kb_log2;
+    TmTree* stree = reinterpret_cast<TmTree*>(smem);                         // [TT] task records
     const int T0 = trees_of(a, 0), T1 = trees_of(a, 1), T2 = t.nm > 2 ? trees_of(a, 2) : 0,
               T3 = t.nm > 2 ? trees_of(a, 3) : 0;
     const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + T3;
-    const int NS = t.nsub;
+    int* stk_b = reinterpret_cast<int*>(stree + TT);                         // [kTmS][NT] record blocks
+    float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
+    float* xs = stk_c + kTmS * NT;                                           // [F + 2][KB] block's features
+    unsigned char* smodel = reinterpret_cast<unsigned char*>(xs + (size_t)(F + 2) * KB);   // [TT] (!FXALL)
+    __shared__ int s_pool[32];                                               // dynamic mode: next task per pool
+    __shared__ int s_fx[4];                                                  // per model: int32 leaves,
+    __shared__ double s_scale[4];                                            // fixed-point scale
+    const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
+    constexpr unsigned kEnt = 4u * NT;                                       // bytes between stack entries
+    const unsigned xs_a = su32(xs);
+    unsigned rs;                                                             // feature row stride (bytes),
+    asm volatile("mov.u32 %0, %1;" : "=r"(rs) : "r"(4u * (unsigned)KB));     // kept in a register
+
+    const int NS = SUB ? t.nsub : 1;
     const long long per_kb = (long long)TT * NS * KB;
     for (int q = threadIdx.x; q < TT; q += NT) {
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
-        stree[q] = make_int2(__ldg(model_of(a, mi).broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3))), mi);
+        const DevModel& d = model_of(a, mi);
+        TmTree r;
+        r.root = __ldg(d.broot + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
+        r.slot_off = t.slot_of[mi] * n_f;
+        r.blocks = d.blocks;
+        stree[q] = r;
+        if (!FXALL) smodel[q] = (unsigned char)mi;
     }
-    if (threadIdx.x < 4) {
+    if (!FXALL && threadIdx.x < 4) {
         const int m = threadIdx.x;
         if (m < 2 || t.nm > 2) {
             const DevModel& d = model_of(a, m);
-            s_blocks[m] = d.blocks;
-            s_slot[m] = t.slot_of[m] * n_f;
             s_fx[m] = d.fx32;
             s_scale[m] = d.fx_scale;
         }
     }
-    __syncthreads();
     const long long r0 = (long long)blockIdx.x * t.n_tasks / gridDim.x;
     const long long r1 = (long long)(blockIdx.x + 1) * t.n_tasks / gridDim.x;
     const int lane = threadIdx.x & 31;
+    const size_t row = (size_t)t.nslot * n_f;                                // D entries per kernel
 
     for (long long s0 = r0; s0 < r1;) {
         const long long kbi = s0 / per_kb;
         const long long s1 = min(r1, (kbi + 1) * per_kb);
         const int kbase = (int)(kbi * KB);                                   // slab-relative
         const int nvalid = min(KB, t.nks - kbase);
-
-        // Static lane streams (large batches): task j (tree j / KB, kernel-in-block j % KB) of the
-        // segment goes to lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same
-        // kernel kk and its trees advance by NT / KB.  Dynamic (t.dyn, batches of a few tasks per
-        // lane): lanes take their first task by thread index and the next ones from a shared
-        // counter, so lanes that drew short walks take the remaining tasks; the lane's feature
-        // column is reloaded when its kernel changes.
+        // the kernel block's static features into shared memory, once per segment, transposed
+        // ([feature][kernel]: lanes on kernels distinct mod 32 read distinct banks); row F + 1 = 0
+        // for folded leaves (row F, the clock, is never read: clock splits take clk)
+        __syncthreads();                                                     // previous segment done
+        const float* gblk = a.features + (t.slab0 + kbase) * F;
+        for (int e = threadIdx.x; e < nvalid * F; e += NT) {
+            const int r = e / F;
+            xs[(e - r * F) * KB + r] = __ldg(gblk + e);
+        }
+        for (int r = threadIdx.x; r < KB; r += NT) xs[(F + 1) * KB + r] = 0.0f;
         const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);
+        // first task of each pool (tasks j = l mod 32) at or after seg0
+        const int base_l = seg0 + (((lane - seg0) % 32) + 32) % 32;
+        if (threadIdx.x < 32) s_pool[lane] = base_l + NT;
+        __syncthreads();
+        // Static lane streams (t.dyn == 0): task j (tree j / KB, kernel-in-block j % KB) of the
+        // segment goes to lane j % 32 of warp (j / 32) % NW, so every task of a lane has the same
+        // kernel and its trees advance by NT / KB.  Dynamic (t.dyn): per-lane-index pools, lane l
+        // of every warp takes the tasks j = l mod 32 in task order from its pool's counter (one
+        // conflict-free shared atomic per task), so the CTA's lanes stay within a few trees (L1-
+        // resident), lanes that drew short walks take the remaining tasks, and the kernels of a
+        // warp's lanes stay distinct mod 32 (conflict-free feature reads: kernel kk sits in bank
+        // kk mod 32 of every feature row).  Either way a task start only sets registers: the
+        // kernel's features are already in shared memory.
         int q;
         if (t.dyn) {
-            __syncthreads();                                                 // previous segment's counter
-            if (threadIdx.x == 0) s_next = seg0 + NT;
-            __syncthreads();
-            q = seg0 + threadIdx.x;
+            q = base_l + 32 * (threadIdx.x >> 5);
         } else {
             const int nw = NT / 32, w = threadIdx.x >> 5;
             const int g0 = seg0 >> 5;
@@ -171,61 +200,54 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
             q = 32 * g + lane;
             if (q < seg0) q += NT;
         }
-        int kk = -1;
-        long long* dbase = t.D;
-        const uint4* blocks = a.ms.blocks;
-        long long* drow = dbase;
+        long long* const dk = t.D + (size_t)kbase * row;                     // the block's D rows
+        long long* drow = dk;
+        const uint4* blocks = nullptr;
         double scale = 1.0;
         bool fxm = true;                                                     // this model's leaves are int32
         int bk = 0, lo = 0, sn = 0, end = n_f;
-        float tmin = CUDART_INF_F;
+        unsigned xb = xs_a;
+        float tmin = CUDART_INF_F, clk = 0.5f;
         long long vprev = 0;
-        bool active = false;
-        // take task offset q if it exists: its kernel's features into the lane column if new
-        auto take = [&](int qq) {
-            while (qq < seg1 && (qq & (KB - 1)) >= nvalid)                   // padding kernels
-                qq = t.dyn ? atomicAdd(&s_next, 1) : qq + NT;
-            q = qq;
-            active = qq < seg1;
-            if (!active) return;
-            const int k2 = qq & (KB - 1);
-            if (k2 != kk) {
-                kk = k2;
-                dbase = t.D + (size_t)(kbase + kk) * t.nslot * n_f;
-                const float* g = a.features + (t.slab0 + kbase + kk) * F;
-                for (int c = 0; c < F; ++c) xcol[(size_t)c * NT] = __ldg(g + c);
-            }
-        };
-        take(q);
-        // start the task at offset q: tree (q / KB) / NS, clock sub-range (q / KB) % NS of this
-        // lane's kernel.  A sub-range [lo, end) walks from the root at clock lo and, at its end,
-        // takes its last value back out at D[end] so the difference arrays stay exact.
-        auto start = [&](int qq) {
-            const int ts = qq >> t.kb_log2;
-            const int tti = NS == 1 ? ts : ts / NS, sub = ts - tti * NS;
-            const int2 ti = stree[tti];
-            bk = ti.x;
-            blocks = s_blocks[ti.y];
-            drow = dbase + s_slot[ti.y];
+        // start the task at offset q (skipping padding kernels of a partial block): tree
+        // (q / KB) / NS, clock sub-range (q / KB) % NS, kernel q % KB.  A sub-range [lo, end)
+        // walks from the root at clock lo and, at its end, takes its last value back out at D[end]
+        // so the difference arrays stay exact.  Returns false when the lane's tasks are exhausted.
+        auto start = [&]() {
+            while (q < seg1 && (q & (KB - 1)) >= nvalid) q = t.dyn ? atomicAdd(&s_pool[lane], 32) : q + NT;
+            if (q >= seg1) return false;
+            const int kk = q & (KB - 1);
+            xb = xs_a + 4u * (unsigned)kk;
+            const int ts = q >> KBL;
+            const int tti = SUB ? ts / NS : ts;
+            const TmTree tr = stree[tti];
+            bk = tr.root;
+            blocks = tr.blocks;
+            drow = dk + (size_t)kk * row + tr.slot_off;
             if (!FXALL) {
-                fxm = s_fx[ti.y] != 0;                                       // as k_cut_blocks converted them
-                scale = s_scale[ti.y];
+                const int mi = smodel[tti];
+                fxm = s_fx[mi] != 0;                                         // as k_cut_blocks converted them
+                scale = s_scale[mi];
             }
-            lo = NS == 1 ? 0 : sub * n_f / NS;                               // n_f <= 4096, NS <= 64
-            end = NS == 1 ? n_f : (sub + 1) * n_f / NS;
-            sts_f(xclk_a, (float)lo + 0.5f);                                 // clock lo enters as lo + 0.5
+            if (SUB) {
+                const int sub = ts - tti * NS;
+                lo = sub * n_f / NS;                                         // n_f <= 4096, NS <= 64
+                end = (sub + 1) * n_f / NS;
+            }
+            clk = (float)lo + 0.5f;                                          // clock lo enters as lo + 0.5
             tmin = CUDART_INF_F;
             sn = 0;
             vprev = 0;
+            return true;
         };
-        if (active) start(q);
+        bool active = start();
         while (active) {                                                     // lanes leave as they finish
             uint4 A, B;
             const int cur = bk;
             ldg_blk256(blocks + 2 * (size_t)cur, A, B);
             float cb;
             bool at_leaf;
-            const unsigned g = tm_step<NT>(A, B, xcol, cb, at_leaf);
+            const unsigned g = tm_step(A, B, xb, rs, clk, cb, at_leaf);
             bk = (int)g;
             if (cb < tmin) {                                                 // new record
                 if (sn < kTmS) {                                             // deeper ones are not kept:
@@ -248,12 +270,13 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                     bk = (int)lds_u(sb_a + kEnt * (unsigned)sn);
                     tmin = sn > 0 ? lds_f(sc_a + kEnt * (unsigned)(sn - 1)) : CUDART_INF_F;
                     lo = hi;
-                    sts_f(xclk_a, (float)hi + 0.5f);
+                    clk = (float)hi + 0.5f;
                 } else {
-                    if (end < n_f)                                           // sub-range end: D[end] -= v
+                    if (SUB && end < n_f)                                    // sub-range end: D[end] -= v
                         atomicAdd(reinterpret_cast<unsigned long long*>(drow + end), (unsigned long long)(-v));
-                    take(t.dyn ? atomicAdd(&s_next, 1) : q + NT);            // next task
-                    if (active) start(q);
+                    q = t.dyn ? atomicAdd(&s_pool[lane], 32) : q + NT;
+                    if (!SUB) lo = 0;
+                    active = start();
                 }
             }
         }

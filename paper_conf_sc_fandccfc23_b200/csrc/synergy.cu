@@ -240,8 +240,10 @@ DevState* dev_state(int dev) {
         if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) == cudaSuccess && v > 0) d.optin = v;
         cudaError_t e = cudaSuccess;
         auto chk = [&e](cudaError_t x) { if (e == cudaSuccess) e = x; };
-        chk(allow_smem(k_tm_walk<kTmNT, true>, d.optin));
-        chk(allow_smem(k_tm_walk<kTmNT, false>, d.optin));
+        chk(allow_smem(k_tm_walk<kTmNT, true, false>, d.optin));
+        chk(allow_smem(k_tm_walk<kTmNT, false, false>, d.optin));
+        chk(allow_smem(k_tm_walk<kTmNT, true, true>, d.optin));
+        chk(allow_smem(k_tm_walk<kTmNT, false, true>, d.optin));
         chk(allow_smem(k_tm_finish, d.optin));
         chk(allow_smem(k_svr<1>, d.optin));
         chk(allow_smem(k_svr<2>, d.optin));
@@ -253,7 +255,7 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_svr<8>, d.optin));
         chk(allow_smem(k_svr_u, d.optin));
         cudaFuncAttributes fa;
-        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false>));
+        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false, true>));
         d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
         if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_finish));
         d.finish_dyn_max = d.optin - (int)fa.sharedSizeBytes;
@@ -454,7 +456,21 @@ constexpr size_t kTmSlabBytes = 48u << 20;   // D bytes per slab (stays L2-resid
 const DevModel& dm_of(const SweepArgs& a, int m) { return m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2]; }
 bool present(const SweepArgs& a, int m) { return m < 2 || a.has_x[m - 2]; }
 
-size_t tm_walk_smem(int F, int tt) { return (size_t)kTmS * kTmNT * 8 + (size_t)(F + 2) * kTmNT * 4 + 16 + (size_t)tt * 8; }
+// k_tm_walk kernels per feature block: a power of two in [32, 256] whose [F + 2][kb] fp32 feature
+// table takes at most 32 KB of shared memory, and no more than the batch needs.
+int tm_kb(int F, long long n_k, long long knob) {
+    const size_t xs = (size_t)(F + 2) * 4;
+    int kb = 256;
+    while (kb > 32 && (xs * kb > 32768 || kb / 2 >= n_k)) kb /= 2;
+    if (knob > 0) {
+        while (kb > 32 && kb > knob) kb /= 2;
+        while (kb < 256 && kb * 2 <= knob) kb *= 2;
+    }
+    return kb;
+}
+size_t tm_walk_smem(int F, int kb, int tt) {
+    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * kTmNT * 8 + (size_t)kb * (F + 2) * 4 + (size_t)tt + 16;
+}
 size_t tm_finish_smem(int nm, int k, int n_f, int xs, int nslot) {
     return (size_t)nm * k * n_f * 12 + (size_t)n_f * 4 + (size_t)k * xs * 4 + 32 + (size_t)k * nslot * n_f * 8;
 }
@@ -472,7 +488,7 @@ bool tm_eligible(const SweepArgs& a, int nm, const DevState* ds) {
         ++nslot;
     }
     if (tt == 0) return false;
-    if (tm_walk_smem(a.F, tt) > (size_t)ds->walk_dyn_max) return false;
+    if (tm_walk_smem(a.F, tm_kb(a.F, a.n_k, knobs().tm_kb.load()), tt) > (size_t)ds->walk_dyn_max) return false;
     return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->finish_dyn_max;
 }
 
@@ -519,14 +535,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     bool fxall = true;                            // every forest has int32 fixed-point leaves
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0 && !dms[m]->fx32) fxall = false;
-    // kernels per feature block: a power of two in [32, 256], F * kb floats of shared memory
-    int kb = 256;
-    while (kb > 32 && ((size_t)F * kb * 4 > 32768 || kb / 2 >= n_k)) kb /= 2;
-    const long long kb_knob = K.tm_kb.load();
-    if (kb_knob > 0) {
-        while (kb > 32 && kb > kb_knob) kb /= 2;
-        while (kb < 256 && kb * 2 <= kb_knob) kb *= 2;
-    }
+    const int kb = tm_kb(F, n_k, K.tm_kb.load());
     t.kb = kb;
     t.kb_log2 = 0;
     while ((1 << t.kb_log2) < kb) ++t.kb_log2;
@@ -571,7 +580,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         return ok();
     }
     const size_t fsmem = fsmem_of(kt);
-    const size_t wsmem = tm_walk_smem(F, tt);
+    const size_t wsmem = tm_walk_smem(F, kb, tt);
     const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : 2LL * ds->sms);
     t.s = a;
     int n = 0;
@@ -601,14 +610,19 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         if (K.tm_nsub.load() >= 1 && K.tm_nsub.load() <= std::min(n_f, 64)) t.nsub = (int)K.tm_nsub.load();
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * t.nsub * kb;
         // a few tasks per lane: dynamic task fetch balances walks of different lengths
-        t.dyn = K.tm_dyn.load() >= 0 ? (K.tm_dyn.load() ? 1 : 0) : (t.n_tasks < 4 * lanes ? 1 : 0);
+        // per-lane-index task pools by default (L1-resident tree window, balanced, conflict-free);
+        // static lane streams on request (tm_dyn = 0)
+        t.dyn = K.tm_dyn.load() >= 0 ? (K.tm_dyn.load() ? 1 : 0) : 1;
         {
             const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
             KernelTimer ktm("k_tm_walk", st);
-            if (fxall)
-                k_tm_walk<kTmNT, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-            else
-                k_tm_walk<kTmNT, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            if (t.nsub == 1) {
+                if (fxall) k_tm_walk<kTmNT, true, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+                else k_tm_walk<kTmNT, false, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            } else {
+                if (fxall) k_tm_walk<kTmNT, true, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+                else k_tm_walk<kTmNT, false, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            }
             e = cudaGetLastError();
         }
         if (e != cudaSuccess) return fail_launch("k_tm_walk launch");

@@ -133,12 +133,14 @@ def test_fuzz_bit_exact(case, variant):
 
 
 def test_path_routing():
-    """Which kernels run: the tree-major pair for in-range forests that fit shared memory, the
-    general exact pair for out-of-range leaves, F beyond k_tm_walk's shared memory, and models
-    without a forest member.  Both paths are checked bit-exact elsewhere."""
+    """Which kernels run: the tree-major pair for in-range forests whose per-tree task table fits
+    shared memory (any F), the general exact pair for out-of-range leaves, 2 x 15000 trees (the
+    tree table exceeds shared memory) and models without a forest member.  Both paths are checked
+    bit-exact elsewhere."""
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
     cases = [(W.fuzz_workload(77, 40, 64, F=4, n_trees=3, max_depth=8), syn.VARIANT_TREE_MAJOR),
-             (W.fuzz_workload(78, 40, 64, F=120, n_trees=3, max_depth=8), syn.VARIANT_GENERAL),
+             (W.fuzz_workload(78, 40, 64, F=200, n_trees=3, max_depth=8), syn.VARIANT_TREE_MAJOR),
+             (W.fuzz_workload(76, 9, 33, F=3, n_trees=15000, max_depth=1, p_leaf=0.0), syn.VARIANT_GENERAL),
              (W.fuzz_workload(79, 40, 64, F=4, n_trees=3, max_depth=4, linear="only"), syn.VARIANT_GENERAL),
              (_stump_models([2.0 ** 60, 100.0, 100.0], [1.0, 2.0]), syn.VARIANT_GENERAL)]
     for w, want in cases:

@@ -46,6 +46,58 @@ __global__ void __launch_bounds__(512, 2) k_scatter32(const uint4* __restrict__ 
     if (acc == 0x9e3779b9u) sink[0] = acc;
 }
 
+// W consecutive 32-byte pieces per load (W = 1, 2, 4: 32 / 64 / 128 bytes, one 128-byte line at
+// most) from random W-aligned positions of the window: is a wider block cheaper per byte?
+template <int W>
+__global__ void __launch_bounds__(512, 2) k_scatter_w(const uint4* __restrict__ buf, unsigned window_blocks,
+                                                      unsigned long long stride_blocks, int iters,
+                                                      unsigned* sink, long long* cycles) {
+    const uint4* base = buf + 2ull * (unsigned long long)(blockIdx.x >> 1) * stride_blocks;
+    unsigned x = (threadIdx.x + 1u) * 2654435761u ^ (blockIdx.x * 40503u);
+    unsigned acc = 0;
+    __syncthreads();
+    const long long t0 = clock64();
+#pragma unroll 4
+    for (int i = 0; i < iters; ++i) {
+        x = x * 1664525u + 1013904223u;
+        const unsigned b = ((x >> 7) & (window_blocks - 1u)) & ~(unsigned)(W - 1);
+#pragma unroll
+        for (int w = 0; w < W; ++w) {
+            uint4 A, B;
+            ldg256(base + 2ull * (b + w), A, B);
+            acc ^= A.x ^ B.w;
+        }
+    }
+    __syncthreads();
+    const long long t1 = clock64();
+    if (threadIdx.x == 0) cycles[blockIdx.x] = t1 - t0;
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
+// Lane pairs: lanes 2i and 2i+1 load the two 32-byte halves of one 64-byte aligned region in the
+// same instruction (one line per pair), as two lanes sharing 64-byte blocks would.
+__global__ void __launch_bounds__(512, 2) k_scatter_pair(const uint4* __restrict__ buf, unsigned window_blocks,
+                                                         unsigned long long stride_blocks, int iters,
+                                                         unsigned* sink, long long* cycles) {
+    const uint4* base = buf + 2ull * (unsigned long long)(blockIdx.x >> 1) * stride_blocks;
+    unsigned x = ((threadIdx.x >> 1) + 1u) * 2654435761u ^ (blockIdx.x * 40503u);
+    unsigned acc = 0;
+    __syncthreads();
+    const long long t0 = clock64();
+#pragma unroll 8
+    for (int i = 0; i < iters; ++i) {
+        x = x * 1664525u + 1013904223u;
+        const unsigned b = (((x >> 7) & (window_blocks - 1u)) & ~1u) + (threadIdx.x & 1u);
+        uint4 A, B;
+        ldg256(base + 2ull * b, A, B);
+        acc ^= A.x ^ B.w;
+    }
+    __syncthreads();
+    const long long t1 = clock64();
+    if (threadIdx.x == 0) cycles[blockIdx.x] = t1 - t0;
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
 __global__ void __launch_bounds__(512, 2) k_smem_read(int iters, unsigned* sink, long long* cycles) {
     extern __shared__ uint4 sm[];                       // 512 x 16 B per CTA (8 KB)
     sm[threadIdx.x] = make_uint4(threadIdx.x, threadIdx.x * 3u, threadIdx.x * 5u, threadIdx.x * 7u);
@@ -136,6 +188,37 @@ int peaks_measure(int device, double* out) {
     out[5] = (double)ctas * nt * siters * 16.0 / (ms * 1e-3);
     out[6] = (double)ctas * nt * siters * 16.0 / sms / c3;
     out[7] = sms;
+    cudaError_t e = cudaGetLastError();
+    cudaFree(buf);
+    cudaFree(sink);
+    cudaFree(cyc);
+    return e == cudaSuccess ? 0 : (int)e;
+}
+
+// Scattered loads of `width` bytes (32, 64, 128; 1 = 32-byte halves of 64-byte regions by lane pairs) over a window of `window_blocks` 32-byte blocks
+// per SM (L1-resident when small): out[0] = bytes/s, out[1] = loads/s (one load = width bytes).
+int peaks_scatter(int device, int width, unsigned window_blocks, int iters, double* out) {
+    if (cudaSetDevice(device) != cudaSuccess) return 1;
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    const int ctas = 2 * sms, nt = 512;
+    uint4* buf = nullptr;
+    unsigned* sink = nullptr;
+    long long* cyc = nullptr;
+    const size_t bytes = (size_t)(ctas / 2 + 1) * window_blocks * 32;
+    if (cudaMalloc(&buf, bytes) != cudaSuccess || cudaMalloc(&sink, 4) != cudaSuccess ||
+        cudaMalloc(&cyc, sizeof(long long) * ctas) != cudaSuccess)
+        return 2;
+    cudaMemset(buf, 1, bytes);
+    float ms = 0.0f;
+    if (width == 32) ms = best_ms([&] { k_scatter_w<1><<<ctas, nt>>>(buf, window_blocks, window_blocks, iters, sink, cyc); }, 5);
+    else if (width == 64) ms = best_ms([&] { k_scatter_w<2><<<ctas, nt>>>(buf, window_blocks, window_blocks, iters, sink, cyc); }, 5);
+    else if (width == 128) ms = best_ms([&] { k_scatter_w<4><<<ctas, nt>>>(buf, window_blocks, window_blocks, iters, sink, cyc); }, 5);
+    else ms = best_ms([&] { k_scatter_pair<<<ctas, nt>>>(buf, window_blocks, window_blocks, iters, sink, cyc); }, 5);   // 2 lanes / 64 B
+    if (width == 1) width = 32;
+    const double loads = (double)ctas * nt * iters;
+    out[0] = loads * width / (ms * 1e-3);
+    out[1] = loads / (ms * 1e-3);
     cudaError_t e = cudaGetLastError();
     cudaFree(buf);
     cudaFree(sink);
