@@ -278,7 +278,8 @@ syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms
  * tests and benchmarks.  Initialised once from the environment (SYNERGY_<KEY upper-case>), then
  * process-wide.  Keys: "algo" (0 automatic, 1 force the general exact kernels), "tm_kb" (k_tm_walk
  * kernels per feature block, 32..256), "tm_ctas", "tm_nsub", "tm_dyn" (-1 automatic), "tm_pdl",
- * "tm_slab", "tm_pipe", "tm_kt", "gen_kt", "svr_splits"; 0 = automatic unless noted.  INVALID_ARG: unknown key. */
+ * "tm_slab", "tm_pipe", "tm_kt", "tm_split" (-1 automatic), "gen_kt", "svr_splits"; 0 = automatic
+ * unless noted.  INVALID_ARG: unknown key. */
 syn_status synergy_config_set(const char *key, int64_t value);
 syn_status synergy_config_get(const char *key, int64_t *value);
 

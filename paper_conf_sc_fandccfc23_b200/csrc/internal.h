@@ -34,6 +34,11 @@ struct DevModel {
     // a root-to-leaf walk of depth D takes max(1, ceil(D / 2)) block loads.
     const uint4* blocks;
     const int* broot;        // [n_trees] root block of each tree
+    // per-tree clock sub-range split for small batches (k_tm_walk unit tables): {first unit of the
+    // tree within the model, sub-ranges}; sub-ranges ~ ceil(expected runs / the model's mean), so
+    // the longest (kernel, tree) walks are cut into pieces of about average length
+    const int2* tsplit;      // [n_trees]
+    int units_split;         // sum of the sub-ranges over the trees
     int bdepth;              // max(1, ceil(depth / 2)) over all trees
     int nblk;                // blocks of all trees (tree t owns [broot[t], broot[t+1] or nblk))
     // exact leaf sums (Q8): every (finite) fp32 leaf v is an integer multiple of 2^-s

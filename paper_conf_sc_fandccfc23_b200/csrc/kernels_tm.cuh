@@ -74,7 +74,9 @@ struct TmArgs {
     int nslot;                   // D slots = models with a forest member
     int slot_of[4];              // model -> D slot, -1 without forest
     int nm;                      // models in the call (2 or 4)
-    int nsub;                    // clock sub-ranges per (kernel, tree) task (small batches)
+    int nsub;                    // smode 1: clock sub-ranges per (kernel, tree) (tiny batches)
+    int smode;                   // units: 0 one per tree, 1 nsub per tree, 2 per-tree split (tsplit)
+    int units;                   // units per kernel block (tasks per kernel)
     int dyn;                     // k_tm_walk: tasks from a shared counter
 };
 
@@ -104,6 +106,8 @@ __device__ __forceinline__ unsigned tm_step(const uint4& A, const uint4& B, unsi
     return l0 ? (l1 ? B.x : B.y) : (l1 ? B.z : B.w);
 }
 
+__device__ __forceinline__ int d0_units(const SweepArgs& a) { return model_of(a, 0).units_split; }
+
 // Per-tree task record in shared memory: everything a task start needs in one 16-byte load.
 struct __align__(16) TmTree {
     int root;            // root block
@@ -112,7 +116,9 @@ struct __align__(16) TmTree {
 };
 
 // FXALL: every forest of the call has int32 fixed-point leaves (no int64 conversion path).
-// SUB: (kernel, tree) tasks are split into clock sub-ranges (t.nsub > 1, tiny batches).
+// SUB: a task is (kernel, unit) with a unit = (tree, clock sub-range [lo, end)) from a unit table
+// in shared memory (t.smode 1: every tree in t.nsub equal sub-ranges, tiny batches; 2: each tree
+// in its tsplit sub-ranges, small batches); otherwise a unit is a whole tree.
 template <int NT, bool FXALL, bool SUB>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
@@ -126,9 +132,11 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     int* stk_b = reinterpret_cast<int*>(stree + TT);                         // [kTmS][NT] record blocks
     float* stk_c = reinterpret_cast<float*>(stk_b + kTmS * NT);              // [kTmS][NT] record cuts
     float* xs = stk_c + kTmS * NT;                                           // [F + 2][KB] block's features
-    unsigned char* smodel = reinterpret_cast<unsigned char*>(xs + (size_t)(F + 2) * KB);   // [TT] (!FXALL)
+    int2* units = reinterpret_cast<int2*>(xs + (size_t)(F + 2) * KB);         // [U] (SUB) {tree, lo | end << 16}
+    unsigned char* smodel = reinterpret_cast<unsigned char*>(units + (SUB ? t.units : 0));   // [TT] (!FXALL)
     __shared__ int s_pool[32];                                               // dynamic mode: next task per pool
-    __shared__ int s_fx[4];                                                  // per model: int32 leaves,
+    __shared__ int s_nblk[4];                                                // per model: blocks in all,
+    __shared__ int s_fx[4];                                                  // int32 leaves,
     __shared__ double s_scale[4];                                            // fixed-point scale
     const unsigned sb_a = su32(stk_b) + 4u * threadIdx.x, sc_a = su32(stk_c) + 4u * threadIdx.x;
     constexpr unsigned kEnt = 4u * NT;                                       // bytes between stack entries
@@ -136,8 +144,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
     unsigned rs;                                                             // feature row stride (bytes),
     asm volatile("mov.u32 %0, %1;" : "=r"(rs) : "r"(4u * (unsigned)KB));     // kept in a register
 
-    const int NS = SUB ? t.nsub : 1;
-    const long long per_kb = (long long)TT * NS * KB;
+    const int U = SUB ? t.units : TT;
+    const long long per_kb = (long long)U * KB;
     for (int q = threadIdx.x; q < TT; q += NT) {
         const int mi = q < c1 ? 0 : q < c2 ? 1 : q < c3 ? 2 : 3;
         const DevModel& d = model_of(a, mi);
@@ -147,11 +155,27 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         r.blocks = d.blocks;
         stree[q] = r;
         if (!FXALL) smodel[q] = (unsigned char)mi;
+        if (SUB) {
+            int u0, ns;
+            if (t.smode == 1) {
+                u0 = q * t.nsub;
+                ns = t.nsub;
+            } else {
+                const int mbase = (mi >= 1 ? d0_units(a) : 0) + (mi >= 2 ? model_of(a, 1).units_split : 0) +
+                                  (mi >= 3 ? model_of(a, 2).units_split : 0);
+                const int2 sp = __ldg(d.tsplit + (q - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
+                u0 = mbase + sp.x;
+                ns = sp.y;
+            }
+            for (int sub = 0; sub < ns; ++sub)
+                units[u0 + sub] = make_int2(q, (sub * n_f / ns) | (((sub + 1) * n_f / ns) << 16));
+        }
     }
-    if (!FXALL && threadIdx.x < 4) {
+    if (threadIdx.x < 4) {
         const int m = threadIdx.x;
         if (m < 2 || t.nm > 2) {
             const DevModel& d = model_of(a, m);
+            s_nblk[m] = d.nblk;
             s_fx[m] = d.fx32;
             s_scale[m] = d.fx_scale;
         }
@@ -177,6 +201,32 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         }
         for (int r = threadIdx.x; r < KB; r += NT) xs[(F + 1) * KB + r] = 0.0f;
         const int seg0 = (int)(s0 - kbi * per_kb), seg1 = (int)(s1 - kbi * per_kb);
+        // pull the blocks of the segment's first trees (at most 8) into L2 with bulk prefetches
+        // (one per model's contiguous tree range), so the first walks of a cold model do not
+        // serialise DRAM misses; later trees of a long range arrive while the first are walked
+        if (threadIdx.x == 0) {
+            const int ta = SUB ? units[seg0 >> KBL].x : seg0 >> KBL;
+            const int tb = min(ta + 7, SUB ? units[(seg1 - 1) >> KBL].x : (seg1 - 1) >> KBL);
+            int u = ta;
+            while (u <= tb) {
+                const int mi = u < c1 ? 0 : u < c2 ? 1 : u < c3 ? 2 : 3;
+                const int mend = mi == 0 ? c1 : mi == 1 ? c2 : mi == 2 ? c3 : TT;   // model's trees end
+                const int v = min(tb + 1, mend);
+                const int b0 = stree[u].root;
+                const int b1 = v < mend ? stree[v].root : s_nblk[mi];
+                if (b1 > b0) {
+                    const char* p = reinterpret_cast<const char*>(stree[u].blocks + 2 * (size_t)b0);
+                    size_t left = (size_t)(b1 - b0) * 32;
+                    while (left > 0) {
+                        const unsigned n = (unsigned)min(left, (size_t)1 << 20);
+                        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(n) : "memory");
+                        p += n;
+                        left -= n;
+                    }
+                }
+                u = v;
+            }
+        }
         // first task of each pool (tasks j = l mod 32) at or after seg0
         const int base_l = seg0 + (((lane - seg0) % 32) + 32) % 32;
         if (threadIdx.x < 32) s_pool[lane] = base_l + NT;
@@ -209,17 +259,19 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         unsigned xb = xs_a;
         float tmin = CUDART_INF_F, clk = 0.5f;
         long long vprev = 0;
-        // start the task at offset q (skipping padding kernels of a partial block): tree
-        // (q / KB) / NS, clock sub-range (q / KB) % NS, kernel q % KB.  A sub-range [lo, end)
-        // walks from the root at clock lo and, at its end, takes its last value back out at D[end]
-        // so the difference arrays stay exact.  Returns false when the lane's tasks are exhausted.
+        // start the task at offset q (skipping padding kernels of a partial block): unit q / KB
+        // (a tree, or a tree's clock sub-range), kernel q % KB.  A sub-range [lo, end) walks from
+        // the root at clock lo and, at its end, takes its last value back out at D[end] so the
+        // difference arrays stay exact.  Returns false when the lane's tasks are exhausted.
         auto start = [&]() {
             while (q < seg1 && (q & (KB - 1)) >= nvalid) q = t.dyn ? atomicAdd(&s_pool[lane], 32) : q + NT;
             if (q >= seg1) return false;
             const int kk = q & (KB - 1);
             xb = xs_a + 4u * (unsigned)kk;
             const int ts = q >> KBL;
-            const int tti = SUB ? ts / NS : ts;
+            int2 un = make_int2(ts, 0);
+            if (SUB) un = units[ts];
+            const int tti = un.x;
             const TmTree tr = stree[tti];
             bk = tr.root;
             blocks = tr.blocks;
@@ -230,9 +282,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
                 scale = s_scale[mi];
             }
             if (SUB) {
-                const int sub = ts - tti * NS;
-                lo = sub * n_f / NS;                                         // n_f <= 4096, NS <= 64
-                end = (sub + 1) * n_f / NS;
+                lo = un.y & 0xffff;
+                end = un.y >> 16;
             }
             clk = (float)lo + 0.5f;                                          // clock lo enters as lo + 0.5
             tmin = CUDART_INF_F;

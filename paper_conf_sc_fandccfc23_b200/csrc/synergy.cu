@@ -173,6 +173,7 @@ struct Knobs {
     std::atomic<long long> tm_kb{0};      // k_tm_walk kernels per feature block (32..256)
     std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default 2 per SM)
     std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
+    std::atomic<long long> tm_split{-1};  // per-tree sub-range split: -1 auto (small batches), 0 off, 1 on
     std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
     std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
@@ -187,7 +188,7 @@ struct KnobName {
     std::atomic<long long>* v;
 };
 const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
-                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
+                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
                            {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
                            {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits}};
 std::once_flag g_knobs_once;
@@ -468,8 +469,9 @@ int tm_kb(int F, long long n_k, long long knob) {
     }
     return kb;
 }
-size_t tm_walk_smem(int F, int kb, int tt) {
-    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * kTmNT * 8 + (size_t)kb * (F + 2) * 4 + (size_t)tt + 16;
+size_t tm_walk_smem(int F, int kb, int tt, int units) {
+    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * kTmNT * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
+           (size_t)tt + 16;
 }
 size_t tm_finish_smem(int nm, int k, int n_f, int xs, int nslot) {
     return (size_t)nm * k * n_f * 12 + (size_t)n_f * 4 + (size_t)k * xs * 4 + 32 + (size_t)k * nslot * n_f * 8;
@@ -488,7 +490,7 @@ bool tm_eligible(const SweepArgs& a, int nm, const DevState* ds) {
         ++nslot;
     }
     if (tt == 0) return false;
-    if (tm_walk_smem(a.F, tm_kb(a.F, a.n_k, knobs().tm_kb.load()), tt) > (size_t)ds->walk_dyn_max) return false;
+    if (tm_walk_smem(a.F, tm_kb(a.F, a.n_k, knobs().tm_kb.load()), tt, 0) > (size_t)ds->walk_dyn_max) return false;
     return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->finish_dyn_max;
 }
 
@@ -580,7 +582,9 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         return ok();
     }
     const size_t fsmem = fsmem_of(kt);
-    const size_t wsmem = tm_walk_smem(F, kb, tt);
+    int usplit = 0;                               // units of the per-tree split (smode 2)
+    for (int m = 0; m < nm; ++m)
+        if (t.slot_of[m] >= 0) usplit += dms[m]->units_split;
     const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : 2LL * ds->sms);
     t.s = a;
     int n = 0;
@@ -606,9 +610,27 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         // adds a root descent, so batches with a task per lane keep whole tasks)
         t.nsub = 1;
         const long long lanes = (long long)ctas * kTmNT;
-        while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8) t.nsub *= 2;
-        if (K.tm_nsub.load() >= 1 && K.tm_nsub.load() <= std::min(n_f, 64)) t.nsub = (int)K.tm_nsub.load();
-        t.n_tasks = (long long)((t.nks + kb - 1) / kb) * tt * t.nsub * kb;
+        while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8 &&
+               tm_walk_smem(F, kb, tt, 2 * tt * t.nsub) <= (size_t)ds->walk_dyn_max)
+            t.nsub *= 2;
+        if (K.tm_nsub.load() >= 1 && K.tm_nsub.load() <= std::min(n_f, 64) &&
+            tm_walk_smem(F, kb, tt, tt * (int)K.tm_nsub.load()) <= (size_t)ds->walk_dyn_max)
+            t.nsub = (int)K.tm_nsub.load();
+        // small batches (2-8 tasks per lane): the longest walks bound the launch's tail, so trees
+        // whose expected run count exceeds the model's mean are split into clock sub-ranges
+        // (smode 2; measured: c5 walk 194 -> 182 us; at ~1 task per lane (c2) every lane is on its
+        // critical path and the extra root descents cost more: 72 -> 76 us, so it stays off there)
+        t.smode = t.nsub > 1 ? 1 : 0;
+        t.units = tt * t.nsub;
+        const long long ksplit = K.tm_split.load();
+        const long long per_lane = (long long)t.nks * tt / std::max<long long>(lanes, 1);   // tasks per lane
+        if (t.smode == 0 && usplit > tt && (ksplit > 0 || (ksplit < 0 && per_lane >= 2 && per_lane < 8)) &&
+            tm_walk_smem(F, kb, tt, usplit) <= (size_t)ds->walk_dyn_max) {
+            t.smode = 2;
+            t.units = usplit;
+        }
+        t.n_tasks = (long long)((t.nks + kb - 1) / kb) * t.units * kb;
+        const size_t wsmem = tm_walk_smem(F, kb, tt, t.smode ? t.units : 0);
         // a few tasks per lane: dynamic task fetch balances walks of different lengths
         // per-lane-index task pools by default (L1-resident tree window, balanced, conflict-free);
         // static lane streams on request (tm_dyn = 0)
@@ -616,7 +638,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         {
             const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
             KernelTimer ktm("k_tm_walk", st);
-            if (t.nsub == 1) {
+            if (t.smode == 0) {
                 if (fxall) k_tm_walk<kTmNT, true, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
                 else k_tm_walk<kTmNT, false, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
             } else {
@@ -1070,6 +1092,49 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         }
     }
 
+    // Per-tree clock sub-range split for small batches (k_tm_walk unit tables): the expected number
+    // of runs (clock intervals sharing a leaf) of a walk over all clocks, with every static split
+    // taken as 50/50: sum over the leaves of 2^-(static splits on the path), counting only leaves
+    // whose clock interval (from the clock-split thresholds on the path) is not empty.  A tree gets
+    // ceil(runs / the model's mean runs) sub-ranges, at most 8.
+    std::vector<int2> tsplit;
+    int units_split = 0;
+    if (d->forest_weight != 0.0) {
+        std::vector<double> cost((size_t)d->n_trees, 0.0);
+        struct Item { int64_t id; double w; float clo, chi; };
+        std::vector<Item> st;
+        double mean = 0.0;
+        for (int t = 0; t < d->n_trees; ++t) {
+            const int64_t b = d->tree_offset[t];
+            st.assign(1, Item{0, 1.0, -INFINITY, INFINITY});
+            double c = 0.0;
+            while (!st.empty()) {
+                const Item it = st.back();
+                st.pop_back();
+                const int32_t f = d->feature[b + it.id];
+                if (f < 0) { c += it.w; continue; }
+                const float thr = d->value[b + it.id];
+                const int32_t l = d->left[b + it.id], r = d->right[b + it.id];
+                if (f == F) {
+                    if (std::min(it.chi, thr) > it.clo) st.push_back({l, it.w, it.clo, std::min(it.chi, thr)});
+                    if (it.chi > std::max(it.clo, thr)) st.push_back({r, it.w, std::max(it.clo, thr), it.chi});
+                } else {
+                    st.push_back({l, 0.5 * it.w, it.clo, it.chi});
+                    st.push_back({r, 0.5 * it.w, it.clo, it.chi});
+                }
+            }
+            cost[t] = std::max(c, 1e-9);
+            mean += cost[t];
+        }
+        mean /= d->n_trees;
+        tsplit.resize(d->n_trees);
+        for (int t = 0; t < d->n_trees; ++t) {
+            const int ns = std::max(1, std::min(8, (int)std::ceil(cost[t] / mean - 1e-9)));
+            tsplit[t] = make_int2(units_split, ns);
+            units_split += ns;
+        }
+    }
+
     // 2-level blocks (see internal.h): built from the validated description, breadth-first
     std::vector<uint4> blocks;
     std::vector<int> broot;
@@ -1151,7 +1216,9 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     const size_t svb = n_sv * d->n_inputs * sizeof(float), dcb = n_sv * sizeof(double);
     const size_t off_sv = off_r + (rb + 255) / 256 * 256, off_dc = off_sv + (svb + 255) / 256 * 256;
     const size_t off_mn = off_dc + (dcb + 255) / 256 * 256, off_sc = off_mn + (lb + 255) / 256 * 256;
-    const size_t total = has_svr ? off_sc + lb : off_r + rb;
+    const size_t off_ts = ((has_svr ? off_sc + lb : off_r + rb) + 255) / 256 * 256;
+    const size_t tsb = std::max<size_t>(tsplit.size(), 1) * sizeof(int2);
+    const size_t total = off_ts + tsb;
     void* mem = nullptr;
     cudaError_t e = cudaMalloc(&mem, total);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(model)");
@@ -1163,6 +1230,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         (e = cudaMemcpy(base + off_l, lw.data(), lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
         (!blocks.empty() && (e = cudaMemcpy(base + off_b, blocks.data(), blocks.size() * sizeof(uint4), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (!broot.empty() && (e = cudaMemcpy(base + off_r, broot.data(), broot.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess) ||
+        (!tsplit.empty() && (e = cudaMemcpy(base + off_ts, tsplit.data(), tsplit.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (has_svr && ((e = cudaMemcpy(base + off_sv, d->sv, svb, cudaMemcpyHostToDevice)) != cudaSuccess ||
                      (e = cudaMemcpy(base + off_dc, d->dual_coef, dcb, cudaMemcpyHostToDevice)) != cudaSuccess ||
                      (e = cudaMemcpy(base + off_mn, d->in_mean, lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
@@ -1194,6 +1262,8 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
     m->dm.bdepth = bdepth;
+    m->dm.tsplit = reinterpret_cast<const int2*>(base + off_ts);
+    m->dm.units_split = units_split;
     m->n_blocks = (long long)(blocks.size() >> 1);
     m->dm.nblk = (int)m->n_blocks;
     m->dm.fx_ok = fx_ok;
