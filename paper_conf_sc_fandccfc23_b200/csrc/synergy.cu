@@ -21,6 +21,7 @@
 #include "kernels.cuh"
 #include "kernels_gen.cuh"
 #include "kernels_svr.cuh"
+#include "kernels_svr_tc.cuh"
 #include "kernels_tm.cuh"
 #include "synergy.h"
 
@@ -180,7 +181,8 @@ struct Knobs {
     std::atomic<long long> tm_pipe{1};    // slab pipeline (finish on a side stream)
     std::atomic<long long> tm_kt{0};      // k_tm_finish kernels per CTA
     std::atomic<long long> gen_kt{0};     // k_gen_finish kernels per CTA
-    std::atomic<long long> svr_splits{0}; // k_svr SV-range splits (0: fill the SMs)
+    std::atomic<long long> svr_splits{0}; // k_svr / k_svr_tc SV-range splits (0: fill the SMs)
+    std::atomic<long long> svr_tc{1};     // SVR contraction on tcgen05 (int8 digit products); 0: fp64 k_svr
 };
 Knobs g_knobs;
 struct KnobName {
@@ -190,7 +192,8 @@ struct KnobName {
 const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
                            {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
                            {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
-                           {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits}};
+                           {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits},
+                           {"svr_tc", &g_knobs.svr_tc}};
 std::once_flag g_knobs_once;
 
 const Knobs& knobs() {
@@ -255,6 +258,7 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_svr<7>, d.optin));
         chk(allow_smem(k_svr<8>, d.optin));
         chk(allow_smem(k_svr_u, d.optin));
+        chk(allow_smem(k_svr_tc, d.optin));
         cudaFuncAttributes fa;
         if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false, true>));
         d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
@@ -759,9 +763,137 @@ cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, cudaStream_t st) {
 
 constexpr size_t kSvrSlabBytes = 256u << 20;   // U scratch per kernel slab
 
+// Tensor-core SVR contraction (kernels_svr_tc.cuh): V tiles of 64 clocks, their digit planes and
+// column exponents once per call; per kernel slab U tiles, row exponents, digit planes, then
+// k_svr_tc over (128-kernel tile, 64-clock tile, SV split).
+syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, long long n_k, int F,
+                          const syn_clocks* clocks, cudaStream_t st, SvrScratch& scr) {
+    scr.st = st;
+    const int n_f = clocks->n_f;
+    const int tn = kTcN, tiles_n = (n_f + tn - 1) / tn;
+    const int n_svp = (dm.n_sv + kTcKC - 1) / kTcKC * kTcKC;
+    const int n_chunks = n_svp / kTcKC;
+    // kernel slabs (multiples of the 128-kernel tile) bound the U scratch (fp64 + 7 digit planes)
+    long long nks = std::max<long long>(kTcM, (long long)(kSvrSlabBytes / ((size_t)n_svp * 16)) / kTcM * kTcM);
+    nks = std::min<long long>(nks, (n_k + kTcM - 1) / kTcM * kTcM);
+    const long long tiles = (std::min(nks, n_k) + kTcM - 1) / kTcM * tiles_n;
+    int splits = (int)std::max<long long>(1, ds->sms / std::max<long long>(tiles, 1));
+    splits = std::min(splits, kSvrMaxSplits);
+    if (knobs().svr_splits.load() > 0) splits = (int)std::min<long long>(knobs().svr_splits.load(), kSvrMaxSplits);
+    splits = std::max(1, std::min(splits, n_chunks));
+    const int cps = (n_chunks + splits - 1) / splits;
+    splits = (n_chunks + cps - 1) / cps;
+    auto al = [](size_t b) { return (b + 255) / 256 * 256; };
+    const size_t pb = (size_t)splits * (size_t)n_k * n_f * sizeof(double);
+    const size_t vb = (size_t)tiles_n * n_svp * tn * sizeof(double);
+    const size_t vqb = (size_t)tiles_n * tn * n_svp * kTcDig;
+    const size_t evb = (size_t)tiles_n * tn * sizeof(int);
+    const size_t ub = (size_t)((nks + kSvrTK - 1) / kSvrTK) * n_svp * kSvrTK * sizeof(double);
+    const size_t uqb = (size_t)((nks + kTcM - 1) / kTcM) * kTcM * n_svp * kTcDig;
+    const size_t eub = (size_t)nks * sizeof(int);
+    const size_t o_v = al(pb), o_vq = o_v + al(vb), o_ev = o_vq + al(vqb), o_u = o_ev + al(evb);
+    const size_t o_uq = o_u + al(ub), o_eu = o_uq + al(uqb), total = o_eu + eub;
+    void* buf = nullptr;
+    syn_status ps = pool_alloc(ds, total, st, &buf, "SVR scratch");
+    if (ps != SYN_OK) return ps;
+    scr.bufs.push_back(buf);
+    char* b = static_cast<char*>(buf);
+    SvrArgs sa;
+    memset(&sa, 0, sizeof sa);
+    sa.features = d_features;
+    sa.n_k = n_k;
+    sa.F = F;
+    sa.freqs = clocks->d_freqs;
+    sa.n_f = n_f;
+    sa.sv = dm.sv;
+    sa.dual = dm.dual;
+    sa.in_mean = dm.in_mean;
+    sa.in_scale = dm.in_scale;
+    sa.gamma = dm.svr_gamma;
+    sa.n_sv = dm.n_sv;
+    sa.n_svp = n_svp;
+    sa.tn = tn;
+    sa.P = reinterpret_cast<double*>(b);
+    sa.Vt = reinterpret_cast<double*>(b + o_v);
+    sa.Ut = reinterpret_cast<double*>(b + o_u);
+    SvrTcArgs ta;
+    memset(&ta, 0, sizeof ta);
+    ta.n_svp = n_svp;
+    ta.Uq = reinterpret_cast<unsigned char*>(b + o_uq);
+    ta.Vq = reinterpret_cast<unsigned char*>(b + o_vq);
+    ta.eU = reinterpret_cast<int*>(b + o_eu);
+    ta.eV = reinterpret_cast<int*>(b + o_ev);
+    ta.P = sa.P;
+    ta.n_k = n_k;
+    ta.n_f = n_f;
+    ta.chunks_per_split = cps;
+    cudaError_t e = cudaSuccess;
+    const long long nv = (long long)tiles_n * n_svp * tn;
+    {
+        KernelTimer kt("k_svr_v", st);
+        k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
+        e = cudaGetLastError();
+    }
+    SvrTcArgs qa = ta;                                  // V: rows = clocks, tiles of 64
+    qa.src = sa.Vt;
+    qa.rows = n_f;
+    qa.tile_rows = kTcN;
+    qa.dst = const_cast<unsigned char*>(ta.Vq);
+    qa.ex = const_cast<int*>(ta.eV);
+    if (e == cudaSuccess) {
+        KernelTimer kt("k_svr_quant", st);
+        k_svr_rowexp<<<(unsigned)((n_f + 255) / 256), 256, 0, st>>>(qa);
+        const long long nq = (long long)tiles_n * kTcN * (n_svp / 16);
+        k_svr_quant<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(qa);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "SVR clock factors");
+    scr.launches += 3;
+    const size_t usmem = (size_t)F * (64 * sizeof(double) + kSvrJC * sizeof(float));
+    if (usmem > (size_t)ds->optin) return fail(SYN_ERR_UNSUPPORTED, "SVR member with %d inputs exceeds shared memory", F + 1);
+    for (long long s0 = 0; s0 < n_k; s0 += nks) {
+        sa.slab0 = s0;
+        sa.nks = (int)std::min<long long>(nks, n_k - s0);
+        const unsigned kts = (unsigned)((sa.nks + kSvrTK - 1) / kSvrTK);
+        {
+            KernelTimer kt("k_svr_u", st);
+            k_svr_u<<<dim3(kts, (unsigned)(n_svp / kSvrJC)), 256, usmem, st>>>(sa);
+            e = cudaGetLastError();
+        }
+        SvrTcArgs ua = ta;                              // U: rows = the slab's kernels, tiles of 128
+        ua.src = sa.Ut;
+        ua.rows = sa.nks;
+        ua.tile_rows = kTcM;
+        ua.dst = const_cast<unsigned char*>(ta.Uq);
+        ua.ex = const_cast<int*>(ta.eU);
+        const int mts = (sa.nks + kTcM - 1) / kTcM;
+        if (e == cudaSuccess) {
+            KernelTimer kt("k_svr_quant", st);
+            k_svr_rowexp<<<(unsigned)((sa.nks + 255) / 256), 256, 0, st>>>(ua);
+            const long long nq = (long long)mts * kTcM * (n_svp / 16);
+            k_svr_quant<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(ua);
+            e = cudaGetLastError();
+        }
+        if (e == cudaSuccess) {
+            SvrTcArgs g = ta;
+            g.slab0 = s0;
+            g.nks = sa.nks;
+            KernelTimer kt("k_svr_tc", st);
+            k_svr_tc<<<dim3((unsigned)mts, (unsigned)tiles_n, (unsigned)splits), kTcThreads, kTcSmem, st>>>(g);
+            e = cudaGetLastError();
+        }
+        if (e != cudaSuccess) return cuda_fail(e, "SVR tensor-core contraction");
+        scr.launches += 4;
+    }
+    dm.svr_p = sa.P;
+    dm.svr_splits = splits;
+    return ok();
+}
+
 syn_status prepare_svr(DevModel& dm, DevState* ds, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
                        cudaStream_t st, SvrScratch& scr) {
     if (dm.svr_weight == 0.0) return ok();
+    if (knobs().svr_tc.load() != 0) return prepare_svr_tc(dm, ds, d_features, n_k, F, clocks, st, scr);
     scr.st = st;
     const int n_f = clocks->n_f;
     const int cpt = std::min(8, (n_f + 31) / 32);

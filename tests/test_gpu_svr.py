@@ -40,6 +40,14 @@ def knobs():
     yield syn.config_set
     syn.config_set("algo", 0)
     syn.config_set("svr_splits", 0)
+    syn.config_set("svr_tc", 1)
+
+
+@pytest.fixture(params=[1, 0], ids=["tcgen05", "fp64"])
+def contraction(request, knobs):
+    """SVR contraction path: tcgen05 int8 digit products (default) or the fp64 k_svr reference."""
+    knobs("svr_tc", request.param)
+    return request.param
 
 
 ALGOS = [0, 1]      # automatic (tree-major for these forests), general exact path
@@ -48,15 +56,16 @@ ALGOS = [0, 1]      # automatic (tree-major for these forests), general exact pa
 @pytest.mark.parametrize("ensemble", [False, True])
 @pytest.mark.parametrize("algo", ALGOS)
 @pytest.mark.parametrize("splits", [0, 1, 5])
-def test_svr_sweep_matches_oracle(knobs, ensemble, algo, splits):
+def test_svr_sweep_matches_oracle(knobs, contraction, ensemble, algo, splits):
     knobs("algo", algo)
     knobs("svr_splits", splits)
     w = W.make_config("c1", models=W.make_models_svr("c1", n_sv=200, ensemble=ensemble))
     ref = oracle.sweep(w.speedup, w.energy, w.features, w.freqs, w.default_idx, w.targets, want_pred=True)
     got = gpu_sweep(w, want_pred=True)
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
-    # k_svr_v + k_svr_u + k_svr + the sweep pair (walk + finish, or forest + finish)
-    assert syn.last_launch()["kernels"] == 5
+    # fp64: k_svr_v + k_svr_u + k_svr + the sweep pair; tcgen05: k_svr_v, V exponents + digits,
+    # k_svr_u, U exponents + digits, k_svr_tc + the sweep pair
+    assert syn.last_launch()["kernels"] == (9 if contraction else 5)
     check_pred(got["S"], ref["S"], "S")
     dE = check_pred(got["E"], ref["E"], "E")
     np.testing.assert_array_equal(got["choice"], oracle.select(got["S"], got["E"], w.default_idx, w.targets))
@@ -64,8 +73,8 @@ def test_svr_sweep_matches_oracle(knobs, ensemble, algo, splits):
     np.testing.assert_array_equal(got["choice"][same], ref["choice"][same])
 
 
-@pytest.mark.parametrize("n_sv", [1, 15, 16, 17, 300])
-def test_svr_ragged_sizes_and_raw_mode(n_sv):
+@pytest.mark.parametrize("n_sv", [1, 15, 16, 17, 63, 64, 65, 300])
+def test_svr_ragged_sizes_and_raw_mode(contraction, n_sv):
     """n_sv around the 16-SV staging chunk, kernels not a multiple of the 64-kernel tile, clocks
     not a multiple of 32; raw outputs (default_idx = -1) and normalised ones."""
     import torch
@@ -109,7 +118,7 @@ def test_svr_sklearn_model_end_to_end():
     check_pred(S.cpu().numpy(), sk.astype(np.float32), "raw SVR vs sklearn", max_frac=1e-2)
 
 
-def test_svr_full_c2_sweep():
+def test_svr_full_c2_sweep(contraction):
     """c2's shapes (1000 kernels x 196 clocks) with a 512-SV energy model, in the launch
     configuration the bench uses for the SVR line."""
     w = W.make_config("c2", models=W.make_models_svr("c2"))
@@ -123,7 +132,7 @@ def test_svr_full_c2_sweep():
     np.testing.assert_array_equal(got["choice"][same], ref["choice"][same])
 
 
-def test_svr_in_four_model_sweep():
+def test_svr_in_four_model_sweep(contraction):
     """Four-model variant with an SVR energy model (Table 2 lists SVR for MIN_ENERGY/ES)."""
     import torch
     from paper_conf_sc_fandccfc23_b200 import synergy as syn
@@ -143,3 +152,23 @@ def test_svr_in_four_model_sweep():
     dE = check_pred(P[1], ref["P"][1], "E")
     same = (dE == 0).all(axis=1)
     np.testing.assert_array_equal(ch[same], ref["choice"][same])
+
+
+def test_tensor_core_contraction_matches_fp64_path(knobs):
+    """The tcgen05 int8 digit-product contraction (kernels_svr_tc.cuh) against the fp64 k_svr
+    reference on c2 shapes with the 512-SV model: raw SVR predictions (fp32) equal or one ulp
+    apart, and the fp64 partial contractions agree to ~2^-40 of the largest term."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.make_config("c2", models=W.make_models_svr("c2"))
+    hm, ck = syn.Model(w.energy), syn.Clocks(w.freqs)
+    f = torch.from_numpy(w.features).cuda()
+    out = {}
+    for tc in (1, 0):
+        knobs("svr_tc", tc)
+        S, E = syn.predict(hm, hm, f, ck, -1)
+        torch.cuda.synchronize()
+        out[tc] = E.cpu().numpy()
+    d = ulp_diff(out[1], out[0])
+    assert d.max() <= 1
+    assert (d == 1).mean() < 1e-3
