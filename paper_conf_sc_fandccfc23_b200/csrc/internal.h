@@ -58,6 +58,7 @@ struct DevModel {
     const double* in_mean;   // [n_inputs]
     const double* in_scale;  // [n_inputs]
     double svr_gamma, svr_b;
+    int svr_eU;              // max_j |dual_j| < 2^svr_eU (k_svr_tc's digit scale)
     // per call (k_svr): svr_splits partial contractions over SV ranges, [svr_splits][n_k][n_f],
     // summed in split order (+ svr_b) by finish_tile
     const double* svr_p;

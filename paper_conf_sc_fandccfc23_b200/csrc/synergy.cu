@@ -259,6 +259,7 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_svr<8>, d.optin));
         chk(allow_smem(k_svr_u, d.optin));
         chk(allow_smem(k_svr_tc, d.optin));
+        chk(allow_smem(k_svr_udig, d.optin));
         cudaFuncAttributes fa;
         if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false, true>));
         d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
@@ -763,18 +764,17 @@ cudaError_t launch_svr_t(const SvrArgs& sa, dim3 grid, cudaStream_t st) {
 
 constexpr size_t kSvrSlabBytes = 256u << 20;   // U scratch per kernel slab
 
-// Tensor-core SVR contraction (kernels_svr_tc.cuh): V tiles of 64 clocks, their digit planes and
-// column exponents once per call; per kernel slab U tiles, row exponents, digit planes, then
-// k_svr_tc over (128-kernel tile, 64-clock tile, SV split).
+// Tensor-core SVR contraction (kernels_svr_tc.cuh): the V digit planes once per call, then per
+// kernel slab the U digit planes and k_svr_tc over (128-kernel tile, 64-clock tile, SV split).
 syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, long long n_k, int F,
                           const syn_clocks* clocks, cudaStream_t st, SvrScratch& scr) {
     scr.st = st;
     const int n_f = clocks->n_f;
-    const int tn = kTcN, tiles_n = (n_f + tn - 1) / tn;
+    const int tiles_n = (n_f + kTcN - 1) / kTcN;
     const int n_svp = (dm.n_sv + kTcKC - 1) / kTcKC * kTcKC;
     const int n_chunks = n_svp / kTcKC;
-    // kernel slabs (multiples of the 128-kernel tile) bound the U scratch (fp64 + 7 digit planes)
-    long long nks = std::max<long long>(kTcM, (long long)(kSvrSlabBytes / ((size_t)n_svp * 16)) / kTcM * kTcM);
+    // kernel slabs (multiples of the 128-kernel tile) bound the U digit planes to kSvrSlabBytes
+    long long nks = std::max<long long>(kTcM, (long long)(kSvrSlabBytes / ((size_t)n_svp * kTcDig)) / kTcM * kTcM);
     nks = std::min<long long>(nks, (n_k + kTcM - 1) / kTcM * kTcM);
     const long long tiles = (std::min(nks, n_k) + kTcM - 1) / kTcM * tiles_n;
     int splits = (int)std::max<long long>(1, ds->sms / std::max<long long>(tiles, 1));
@@ -785,21 +785,17 @@ syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, l
     splits = (n_chunks + cps - 1) / cps;
     auto al = [](size_t b) { return (b + 255) / 256 * 256; };
     const size_t pb = (size_t)splits * (size_t)n_k * n_f * sizeof(double);
-    const size_t vb = (size_t)tiles_n * n_svp * tn * sizeof(double);
-    const size_t vqb = (size_t)tiles_n * tn * n_svp * kTcDig;
-    const size_t evb = (size_t)tiles_n * tn * sizeof(int);
-    const size_t ub = (size_t)((nks + kSvrTK - 1) / kSvrTK) * n_svp * kSvrTK * sizeof(double);
-    const size_t uqb = (size_t)((nks + kTcM - 1) / kTcM) * kTcM * n_svp * kTcDig;
-    const size_t eub = (size_t)nks * sizeof(int);
-    const size_t o_v = al(pb), o_vq = o_v + al(vb), o_ev = o_vq + al(vqb), o_u = o_ev + al(evb);
-    const size_t o_uq = o_u + al(ub), o_eu = o_uq + al(uqb), total = o_eu + eub;
+    const size_t vqb = (size_t)tiles_n * n_chunks * kTcBBytes;
+    const size_t uqb = (size_t)((nks + kTcM - 1) / kTcM) * n_chunks * kTcABytes;
+    const size_t o_vq = al(pb), o_uq = o_vq + al(vqb), total = o_uq + uqb;
     void* buf = nullptr;
     syn_status ps = pool_alloc(ds, total, st, &buf, "SVR scratch");
     if (ps != SYN_OK) return ps;
     scr.bufs.push_back(buf);
     char* b = static_cast<char*>(buf);
-    SvrArgs sa;
-    memset(&sa, 0, sizeof sa);
+    SvrTcArgs ta;
+    memset(&ta, 0, sizeof ta);
+    SvrArgs& sa = ta.s;
     sa.features = d_features;
     sa.n_k = n_k;
     sa.F = F;
@@ -812,78 +808,37 @@ syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, l
     sa.gamma = dm.svr_gamma;
     sa.n_sv = dm.n_sv;
     sa.n_svp = n_svp;
-    sa.tn = tn;
     sa.P = reinterpret_cast<double*>(b);
-    sa.Vt = reinterpret_cast<double*>(b + o_v);
-    sa.Ut = reinterpret_cast<double*>(b + o_u);
-    SvrTcArgs ta;
-    memset(&ta, 0, sizeof ta);
-    ta.n_svp = n_svp;
-    ta.Uq = reinterpret_cast<unsigned char*>(b + o_uq);
     ta.Vq = reinterpret_cast<unsigned char*>(b + o_vq);
-    ta.eU = reinterpret_cast<int*>(b + o_eu);
-    ta.eV = reinterpret_cast<int*>(b + o_ev);
-    ta.P = sa.P;
-    ta.n_k = n_k;
-    ta.n_f = n_f;
+    ta.Uq = reinterpret_cast<unsigned char*>(b + o_uq);
+    ta.eU = dm.svr_eU;
     ta.chunks_per_split = cps;
     cudaError_t e = cudaSuccess;
-    const long long nv = (long long)tiles_n * n_svp * tn;
     {
-        KernelTimer kt("k_svr_v", st);
-        k_svr_v<<<(unsigned)((nv + 255) / 256), 256, 0, st>>>(sa);
+        KernelTimer kt("k_svr_vdig", st);
+        k_svr_vdig<<<dim3((unsigned)tiles_n, (unsigned)n_chunks), 2 * kTcN, 0, st>>>(ta);
         e = cudaGetLastError();
     }
-    SvrTcArgs qa = ta;                                  // V: rows = clocks, tiles of 64
-    qa.src = sa.Vt;
-    qa.rows = n_f;
-    qa.tile_rows = kTcN;
-    qa.dst = const_cast<unsigned char*>(ta.Vq);
-    qa.ex = const_cast<int*>(ta.eV);
-    if (e == cudaSuccess) {
-        KernelTimer kt("k_svr_quant", st);
-        k_svr_rowexp<<<(unsigned)((n_f + 255) / 256), 256, 0, st>>>(qa);
-        const long long nq = (long long)tiles_n * kTcN * (n_svp / 16);
-        k_svr_quant<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(qa);
-        e = cudaGetLastError();
-    }
-    if (e != cudaSuccess) return cuda_fail(e, "SVR clock factors");
-    scr.launches += 3;
-    const size_t usmem = (size_t)F * (64 * sizeof(double) + kSvrJC * sizeof(float));
+    if (e != cudaSuccess) return cuda_fail(e, "k_svr_vdig launch");
+    scr.launches += 1;
+    const size_t usmem = (size_t)kTcM * (F + 1) * sizeof(double) + (size_t)kTcKC * F * sizeof(float);
     if (usmem > (size_t)ds->optin) return fail(SYN_ERR_UNSUPPORTED, "SVR member with %d inputs exceeds shared memory", F + 1);
     for (long long s0 = 0; s0 < n_k; s0 += nks) {
         sa.slab0 = s0;
         sa.nks = (int)std::min<long long>(nks, n_k - s0);
-        const unsigned kts = (unsigned)((sa.nks + kSvrTK - 1) / kSvrTK);
-        {
-            KernelTimer kt("k_svr_u", st);
-            k_svr_u<<<dim3(kts, (unsigned)(n_svp / kSvrJC)), 256, usmem, st>>>(sa);
-            e = cudaGetLastError();
-        }
-        SvrTcArgs ua = ta;                              // U: rows = the slab's kernels, tiles of 128
-        ua.src = sa.Ut;
-        ua.rows = sa.nks;
-        ua.tile_rows = kTcM;
-        ua.dst = const_cast<unsigned char*>(ta.Uq);
-        ua.ex = const_cast<int*>(ta.eU);
         const int mts = (sa.nks + kTcM - 1) / kTcM;
-        if (e == cudaSuccess) {
-            KernelTimer kt("k_svr_quant", st);
-            k_svr_rowexp<<<(unsigned)((sa.nks + 255) / 256), 256, 0, st>>>(ua);
-            const long long nq = (long long)mts * kTcM * (n_svp / 16);
-            k_svr_quant<<<(unsigned)((nq + 255) / 256), 256, 0, st>>>(ua);
+        {
+            KernelTimer kt("k_svr_udig", st);
+            k_svr_udig<<<dim3((unsigned)mts, (unsigned)n_chunks), 256, usmem, st>>>(ta);
             e = cudaGetLastError();
         }
         if (e == cudaSuccess) {
-            SvrTcArgs g = ta;
-            g.slab0 = s0;
-            g.nks = sa.nks;
             KernelTimer kt("k_svr_tc", st);
-            k_svr_tc<<<dim3((unsigned)mts, (unsigned)tiles_n, (unsigned)splits), kTcThreads, kTcSmem, st>>>(g);
+            k_svr_tc<<<dim3((unsigned)mts, (unsigned)tiles_n, (unsigned)splits), kTcThreads, kTcSmem, st>>>(ta);
             e = cudaGetLastError();
         }
         if (e != cudaSuccess) return cuda_fail(e, "SVR tensor-core contraction");
-        scr.launches += 4;
+        scr.launches += 2;
     }
     dm.svr_p = sa.P;
     dm.svr_splits = splits;
@@ -893,7 +848,8 @@ syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, l
 syn_status prepare_svr(DevModel& dm, DevState* ds, const float* d_features, long long n_k, int F, const syn_clocks* clocks,
                        cudaStream_t st, SvrScratch& scr) {
     if (dm.svr_weight == 0.0) return ok();
-    if (knobs().svr_tc.load() != 0) return prepare_svr_tc(dm, ds, d_features, n_k, F, clocks, st, scr);
+    // the tensor-core path keeps every level accumulator exact in int32 for n_sv <= 16384
+    if (knobs().svr_tc.load() != 0 && dm.n_sv <= 16384) return prepare_svr_tc(dm, ds, d_features, n_k, F, clocks, st, scr);
     scr.st = st;
     const int n_f = clocks->n_f;
     const int cpt = std::min(8, (n_f + 31) / 32);
@@ -1412,6 +1368,11 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         m->dm.in_scale = reinterpret_cast<const double*>(base + off_sc);
         m->dm.svr_gamma = d->svr_gamma;
         m->dm.svr_b = d->svr_intercept;
+        double mx = 0.0;
+        for (int j = 0; j < d->n_sv; ++j) mx = std::max(mx, std::fabs(d->dual_coef[j]));
+        int e = 0;
+        if (mx > 0.0) std::frexp(mx, &e);                  // mx in [2^(e-1), 2^e)
+        m->dm.svr_eU = e;
     }
     m->dm.svr_p = nullptr;
     m->dm.svr_splits = 0;
