@@ -44,15 +44,26 @@ def main():
              W.fuzz_workload(1004, 23, 196, F=4, n_trees=5, max_depth=14, p_freq=0.9, p_leaf=0.05)]
     if mode == "full":
         cases += [W.make_config("c2"), W.fuzz_workload(1005, 600, 64, F=5, n_trees=4, max_depth=9, linear="both")]
+    cases.append(W.make_config("c1", models=W.make_models_svr("c1", n_sv=100, ensemble=True)))
+    cases.append(W.fuzz_workload(1007, 9, 33, F=3, n_trees=4, max_depth=5, linear="only"))
     for w in cases:
         run(w)
         print("ok", w.name, w.n_kernels, w.n_freqs, flush=True)
+    syn.config_set("svr_tc", 0)                              # the fp64 SVR reference path too
+    run(W.make_config("c1", models=W.make_models_svr("c1", n_sv=100)))
+    syn.config_set("svr_tc", 1)
+    syn.config_set("algo", 1)                                # the general exact path on c1
+    run(W.make_config("c1"))
+    syn.config_set("algo", 0)
+    print("ok svr fp64 + general path", flush=True)
     if mode == "full":
-        os.environ["SYNERGY_TM_SLAB"] = "64"
+        syn.config_set("tm_slab", 64)
+        syn.config_set("tm_kb", 32)
         w = W.fuzz_workload(1006, 300, 128, F=12, n_trees=3, max_depth=6)
         run(w)
         print("ok slab pipeline", flush=True)
-        os.environ.pop("SYNERGY_TM_SLAB")
+        syn.config_set("tm_slab", 0)
+        syn.config_set("tm_kb", 0)
         s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
         w = W.make_config("c1")
         with torch.cuda.stream(s1):
