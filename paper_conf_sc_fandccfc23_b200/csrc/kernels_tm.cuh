@@ -52,7 +52,6 @@
 namespace syn {
 
 constexpr int kTmS = 6;          // record-stack entries per lane (a depth-12 path has <= 6 blocks)
-constexpr int kTmNT = 512;       // k_tm_walk threads per CTA (2 CTAs per SM)
 
 // Clock-cut block words (k_cut_blocks output; the layout of internal.h with two additions):
 //   word 3 bits 28/29/30: node / child 0 / child 1 splits on the clock (code == F)

@@ -175,6 +175,7 @@ struct Knobs {
     std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default 2 per SM)
     std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
     std::atomic<long long> tm_split{-1};  // per-tree sub-range split: -1 auto (small batches), 0 off, 1 on
+    std::atomic<long long> tm_nt{512};    // k_tm_walk threads per CTA: 512 or 1024
     std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
     std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
@@ -190,7 +191,7 @@ struct KnobName {
     std::atomic<long long>* v;
 };
 const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
-                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
+                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_nt", &g_knobs.tm_nt}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
                            {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
                            {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits},
                            {"svr_tc", &g_knobs.svr_tc}};
@@ -244,10 +245,14 @@ DevState* dev_state(int dev) {
         if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) == cudaSuccess && v > 0) d.optin = v;
         cudaError_t e = cudaSuccess;
         auto chk = [&e](cudaError_t x) { if (e == cudaSuccess) e = x; };
-        chk(allow_smem(k_tm_walk<kTmNT, true, false>, d.optin));
-        chk(allow_smem(k_tm_walk<kTmNT, false, false>, d.optin));
-        chk(allow_smem(k_tm_walk<kTmNT, true, true>, d.optin));
-        chk(allow_smem(k_tm_walk<kTmNT, false, true>, d.optin));
+        chk(allow_smem(k_tm_walk<512, true, false>, d.optin));
+        chk(allow_smem(k_tm_walk<512, false, false>, d.optin));
+        chk(allow_smem(k_tm_walk<512, true, true>, d.optin));
+        chk(allow_smem(k_tm_walk<512, false, true>, d.optin));
+        chk(allow_smem(k_tm_walk<1024, true, false>, d.optin));
+        chk(allow_smem(k_tm_walk<1024, false, false>, d.optin));
+        chk(allow_smem(k_tm_walk<1024, true, true>, d.optin));
+        chk(allow_smem(k_tm_walk<1024, false, true>, d.optin));
         chk(allow_smem(k_tm_finish, d.optin));
         chk(allow_smem(k_svr<1>, d.optin));
         chk(allow_smem(k_svr<2>, d.optin));
@@ -261,7 +266,7 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_svr_tc, d.optin));
         chk(allow_smem(k_svr_udig, d.optin));
         cudaFuncAttributes fa;
-        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<kTmNT, false, true>));
+        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_walk<1024, false, true>));
         d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
         if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_finish));
         d.finish_dyn_max = d.optin - (int)fa.sharedSizeBytes;
@@ -474,8 +479,11 @@ int tm_kb(int F, long long n_k, long long knob) {
     }
     return kb;
 }
+// k_tm_walk threads per CTA: 512 (two CTAs per SM) or 1024 (one CTA per SM: one tree window and
+// one feature table per SM instead of two)
+int tm_nt() { return knobs().tm_nt.load() == 1024 ? 1024 : 512; }
 size_t tm_walk_smem(int F, int kb, int tt, int units) {
-    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * kTmNT * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
+    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * tm_nt() * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
            (size_t)tt + 16;
 }
 size_t tm_finish_smem(int nm, int k, int n_f, int xs, int nslot) {
@@ -590,7 +598,8 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     int usplit = 0;                               // units of the per-tree split (smode 2)
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0) usplit += dms[m]->units_split;
-    const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : 2LL * ds->sms);
+    const int NTW = tm_nt();
+    const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : (2048LL / NTW) * ds->sms);
     t.s = a;
     int n = 0;
     int slab = 0;
@@ -614,7 +623,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         // tasks than resident lanes (at most 8 sub-ranges of at least 8 clocks; each sub-range
         // adds a root descent, so batches with a task per lane keep whole tasks)
         t.nsub = 1;
-        const long long lanes = (long long)ctas * kTmNT;
+        const long long lanes = (long long)ctas * NTW;
         while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8 &&
                tm_walk_smem(F, kb, tt, 2 * tt * t.nsub) <= (size_t)ds->walk_dyn_max)
             t.nsub *= 2;
@@ -643,12 +652,16 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         {
             const long long g = std::max<long long>(1, std::min<long long>(ctas, (t.n_tasks + 255) / 256));
             KernelTimer ktm("k_tm_walk", st);
-            if (t.smode == 0) {
-                if (fxall) k_tm_walk<kTmNT, true, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-                else k_tm_walk<kTmNT, false, false><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-            } else {
-                if (fxall) k_tm_walk<kTmNT, true, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
-                else k_tm_walk<kTmNT, false, true><<<(unsigned)g, kTmNT, wsmem, st>>>(t);
+            const int cls = (fxall ? 1 : 0) + (t.smode ? 2 : 0) + (NTW == 1024 ? 4 : 0);
+            switch (cls) {
+                case 0: k_tm_walk<512, false, false><<<(unsigned)g, 512, wsmem, st>>>(t); break;
+                case 1: k_tm_walk<512, true, false><<<(unsigned)g, 512, wsmem, st>>>(t); break;
+                case 2: k_tm_walk<512, false, true><<<(unsigned)g, 512, wsmem, st>>>(t); break;
+                case 3: k_tm_walk<512, true, true><<<(unsigned)g, 512, wsmem, st>>>(t); break;
+                case 4: k_tm_walk<1024, false, false><<<(unsigned)g, 1024, wsmem, st>>>(t); break;
+                case 5: k_tm_walk<1024, true, false><<<(unsigned)g, 1024, wsmem, st>>>(t); break;
+                case 6: k_tm_walk<1024, false, true><<<(unsigned)g, 1024, wsmem, st>>>(t); break;
+                default: k_tm_walk<1024, true, true><<<(unsigned)g, 1024, wsmem, st>>>(t); break;
             }
             e = cudaGetLastError();
         }
@@ -1028,7 +1041,8 @@ syn_status run_sweep(const syn_model* const* models, int nm, const float* d_feat
     if (tm) {
         ss = run_tm(a, nm, const_cast<syn_model* const*>(models), clocks, st, ds, false, &nl);
         if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, std::min<long long>(2LL * ds->sms, n_k), kTmNT, kVarTm};
+        g_last = {nl + scr.launches, n_k * (long long)n_f, std::min<long long>((2048LL / tm_nt()) * ds->sms, n_k),
+                  tm_nt(), kVarTm};
         return ok();
     }
     ss = run_gen(a, nm, st, ds, &nl);
