@@ -175,7 +175,7 @@ struct Knobs {
     std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default 2 per SM)
     std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
     std::atomic<long long> tm_split{-1};  // per-tree sub-range split: -1 auto (small batches), 0 off, 1 on
-    std::atomic<long long> tm_nt{512};    // k_tm_walk threads per CTA: 512 or 1024
+    std::atomic<long long> tm_nt{0};      // k_tm_walk threads per CTA: 0 automatic, 512 or 1024
     std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
     std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
@@ -479,11 +479,16 @@ int tm_kb(int F, long long n_k, long long knob) {
     }
     return kb;
 }
-// k_tm_walk threads per CTA: 512 (two CTAs per SM) or 1024 (one CTA per SM: one tree window and
-// one feature table per SM instead of two)
-int tm_nt() { return knobs().tm_nt.load() == 1024 ? 1024 : 512; }
-size_t tm_walk_smem(int F, int kb, int tt, int units) {
-    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * tm_nt() * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
+// k_tm_walk threads per CTA: 1024 (one CTA per SM: one tree window and one feature table per SM
+// instead of two; measured c3 walk 2.62 -> 2.51 ms per slab) for large batches, 512 (two CTAs per
+// SM) when a lane has only a few tasks (c2 72 -> 92 us and c5 181 -> 198 us with 1024)
+int tm_nt(long long slab_tasks, int sms) {
+    const long long k = knobs().tm_nt.load();
+    if (k == 512 || k == 1024) return (int)k;
+    return slab_tasks >= 8LL * 1024 * sms ? 1024 : 512;
+}
+size_t tm_walk_smem(int F, int kb, int tt, int units, int nt = 1024) {
+    return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * nt * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
            (size_t)tt + 16;
 }
 size_t tm_finish_smem(int nm, int k, int n_f, int xs, int nslot) {
@@ -598,8 +603,8 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     int usplit = 0;                               // units of the per-tree split (smode 2)
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0) usplit += dms[m]->units_split;
-    const int NTW = tm_nt();
-    const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : (2048LL / NTW) * ds->sms);
+    const int NTW = tm_nt((long long)nks * tt, ds->sms);
+    const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : (1024LL / NTW) * ds->sms);
     t.s = a;
     int n = 0;
     int slab = 0;
@@ -644,7 +649,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             t.units = usplit;
         }
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * t.units * kb;
-        const size_t wsmem = tm_walk_smem(F, kb, tt, t.smode ? t.units : 0);
+        const size_t wsmem = tm_walk_smem(F, kb, tt, t.smode ? t.units : 0, NTW);
         // a few tasks per lane: dynamic task fetch balances walks of different lengths
         // per-lane-index task pools by default (L1-resident tree window, balanced, conflict-free);
         // static lane streams on request (tm_dyn = 0)
@@ -1041,8 +1046,7 @@ syn_status run_sweep(const syn_model* const* models, int nm, const float* d_feat
     if (tm) {
         ss = run_tm(a, nm, const_cast<syn_model* const*>(models), clocks, st, ds, false, &nl);
         if (ss != SYN_OK) return ss;
-        g_last = {nl + scr.launches, n_k * (long long)n_f, std::min<long long>((2048LL / tm_nt()) * ds->sms, n_k),
-                  tm_nt(), kVarTm};
+        g_last = {nl + scr.launches, n_k * (long long)n_f, 0, 0, kVarTm};
         return ok();
     }
     ss = run_gen(a, nm, st, ds, &nl);
