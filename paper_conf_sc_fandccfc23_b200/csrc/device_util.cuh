@@ -38,12 +38,6 @@ __device__ __forceinline__ uint2 ldg_node(const uint2* p) {
     return r;
 }
 
-__device__ __forceinline__ unsigned lanemask_lt() {
-    unsigned r;
-    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
-    return r;
-}
-
 // Model m of a call: 0 speedup, 1 energy, 2 direct EDP, 3 direct ED2P (four-model variant).
 __device__ __forceinline__ const DevModel& model_of(const SweepArgs& a, int m) {
     return m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2];

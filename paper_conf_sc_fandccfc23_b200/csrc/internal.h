@@ -39,7 +39,6 @@ struct DevModel {
     // the longest (kernel, tree) walks are cut into pieces of about average length
     const int2* tsplit;      // [n_trees]
     int units_split;         // sum of the sub-ranges over the trees
-    int bdepth;              // max(1, ceil(depth / 2)) over all trees
     int nblk;                // blocks of all trees (tree t owns [broot[t], broot[t+1] or nblk))
     // exact leaf sums (Q8): every (finite) fp32 leaf v is an integer multiple of 2^-s
     // (s from the smallest leaf ulp).  fx_ok: n_trees * max|v| * 2^s < 2^62, so v * 2^s is an

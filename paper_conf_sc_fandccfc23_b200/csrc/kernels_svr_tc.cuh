@@ -163,7 +163,9 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant_
     unsigned long long* empty = full + kTcStages;
     unsigned long long* accb = empty + kTcStages;
     unsigned* tmem_slot = reinterpret_cast<unsigned*>(accb + 1);
-    const int mt = blockIdx.x, nt = blockIdx.y;
+    // clock tiles vary fastest across the grid, so the CTAs that share a kernel tile's U digits run
+    // together and read them from DRAM once (L2 serves the others)
+    const int nt = blockIdx.x, mt = blockIdx.y;
     const int n_chunks = a.n_svp / kTcKC;
     const int c0 = blockIdx.z * t.chunks_per_split;
     const int nch = min(t.chunks_per_split, n_chunks - c0);

@@ -176,6 +176,7 @@ struct Knobs {
     std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
     std::atomic<long long> tm_split{-1};  // per-tree sub-range split: -1 auto (small batches), 0 off, 1 on
     std::atomic<long long> tm_nt{0};      // k_tm_walk threads per CTA: 0 automatic, 512 or 1024
+    std::atomic<long long> split_piece{4};// model create: sub-range target cost, in quarters of the mean
     std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
     std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
@@ -191,7 +192,7 @@ struct KnobName {
     std::atomic<long long>* v;
 };
 const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
-                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_nt", &g_knobs.tm_nt}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
+                           {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_nt", &g_knobs.tm_nt}, {"split_piece", &g_knobs.split_piece}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
                            {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
                            {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits},
                            {"svr_tc", &g_knobs.svr_tc}};
@@ -852,7 +853,7 @@ syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, l
         }
         if (e == cudaSuccess) {
             KernelTimer kt("k_svr_tc", st);
-            k_svr_tc<<<dim3((unsigned)mts, (unsigned)tiles_n, (unsigned)splits), kTcThreads, kTcSmem, st>>>(ta);
+            k_svr_tc<<<dim3((unsigned)tiles_n, (unsigned)mts, (unsigned)splits), kTcThreads, kTcSmem, st>>>(ta);
             e = cudaGetLastError();
         }
         if (e != cudaSuccess) return cuda_fail(e, "SVR tensor-core contraction");
@@ -1235,7 +1236,8 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         mean /= d->n_trees;
         tsplit.resize(d->n_trees);
         for (int t = 0; t < d->n_trees; ++t) {
-            const int ns = std::max(1, std::min(8, (int)std::ceil(cost[t] / mean - 1e-9)));
+            const double piece = mean * (double)std::max<long long>(1, knobs().split_piece.load()) / 4.0;
+            const int ns = std::max(1, std::min(8, (int)std::ceil(cost[t] / piece - 1e-9)));
             tsplit[t] = make_int2(units_split, ns);
             units_split += ns;
         }
@@ -1244,7 +1246,6 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     // 2-level blocks (see internal.h): built from the validated description, breadth-first
     std::vector<uint4> blocks;
     std::vector<int> broot;
-    int bdepth = 1;
     if (d->forest_weight != 0.0) {
         broot.resize(d->n_trees);
         std::vector<int64_t> q;
@@ -1305,7 +1306,6 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
                 blocks[2 * qb[p]] = make_uint4(w[0], w[1], w[2], w[3]);
                 blocks[2 * qb[p] + 1] = make_uint4(w[4], w[5], w[6], w[7]);
             }
-            bdepth = std::max(bdepth, (trees[t].y + 1) / 2);
         }
     }
 
@@ -1367,7 +1367,6 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.depth = max_depth;
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
-    m->dm.bdepth = bdepth;
     m->dm.tsplit = reinterpret_cast<const int2*>(base + off_ts);
     m->dm.units_split = units_split;
     m->n_blocks = (long long)(blocks.size() >> 1);
