@@ -504,14 +504,14 @@ def main():
                     "onchip_peaks_measured": onchip, "hbm": hbm, "per_kernel": per_kernel}
 
     if "k_svr_tc" in ktimes:
-        # the SVR contraction on tcgen05: the int8 digit products it issues (36 digit pairs x
+        # the SVR contraction on tcgen05: the int8 digit products it issues (28 digit pairs x
         # 2 * M * N * K per tile, padded tiles) against the int8 dense peak (measured bf16 x 2, the
         # nominal int8 / bf16 ratio 4.5 / 2.25 PFLOP/s)
         tc_s = ktimes["k_svr_tc"][0] / ktimes["k_svr_tc"][1] / 1e3
         per_step = max(1.0, ktimes["k_svr_tc"][1] / K)
         n_k_l = evals_step // n_f
         n_svp = -(-en_spec.n_sv // 32) * 32
-        ops = 36 * 2.0 * (-(-n_k_l // 128) * 128) * (-(-n_f // 64) * 64) * n_svp / per_step
+        ops = 28 * 2.0 * (-(-n_k_l // 128) * 128) * (-(-n_f // 64) * 64) * n_svp / per_step
         roofline["svr_contraction"] = {
             "bound": "tensor", "kernel": "k_svr_tc", "kernel_ms": tc_s * 1e3, "achieved": ops / tc_s / 1e12,
             "peak": 2.0 * peaks["bf16_tflops"], "unit": "TOP/s (int8)",

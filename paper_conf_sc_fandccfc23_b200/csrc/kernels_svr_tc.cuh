@@ -7,15 +7,16 @@
 // the 1e-5 bar.  This path uses exact integer tensor-core products instead (an Ozaki-style split):
 //
 //   * U is scaled by 2^-eU (eU = the exponent of max_j |dual_j|, fixed per model: |U| <= max|dual|
-//     < 2^eU) and V by 2^-1 (V <= 1 < 2^1), so both lie in (-1, 1), and each value is written as 8
-//     signed 7-bit digits, x = sum_p d_p 2^-7(p+1), |d_p| <= 127, truncated below 2^-56;
-//   * U V = 2^(eU + 1) sum_{p,q} 2^-7(p+q+2) (D_p E_q), and each digit product D_p E_q is an int8 x
-//     int8 GEMM with exact int32 accumulation (tcgen05.mma kind::i8; |sum| <= 127^2 * n_sv * 8 <
-//     2^31 for n_sv <= 16384).  Products of equal level L = p + q share one TMEM accumulator (8
-//     levels x 64 columns = the SM's 512 TMEM columns); levels L >= 8 are dropped;
-//   * the epilogue reads the 8 level accumulators (tcgen05.ld), sums 2^-7(L+2) acc_L in fp64 and
-//     scales by 2^(eU + 1).  Digit truncation and the dropped levels change each term by at most
-//     2^-53 max_j|dual_j| (both factors' scales are powers of two), so the value is within
+//     < 2^eU) and V by 2^-1 (V <= 1 < 2^1), so both lie in (-1, 1); each scaled value x becomes the
+//     integer X = round(x 2^54) written with 7 balanced base-256 digits, X = sum_p d_p 256^(6-p),
+//     d_p in [-128, 127] (signed bytes), |x - X 2^-54| <= 2^-55;
+//   * U V = 2^(eU + 1 - 108) sum_{p,q} 256^(12-p-q) (D_p E_q), and each digit product D_p E_q is an
+//     int8 x int8 GEMM with exact int32 accumulation (tcgen05.mma kind::i8; |sum| <= 128^2 * n_sv
+//     * 7 < 2^31 for n_sv <= 16384).  Products of equal level L = p + q share one TMEM accumulator
+//     (7 levels x 64 columns); levels L >= 7 are dropped (the 28 pairs with L <= 6 are kept);
+//   * the epilogue reads the 7 level accumulators (tcgen05.ld), sums 2^-(8L+12) acc_L in fp64 and
+//     scales by 2^(eU + 1).  Digit rounding and the dropped levels change each term by at most
+//     about 2^-53 max_j|dual_j| (both factors' scales are powers of two), so the value is within
 //     n_sv 2^-53 max_j|dual_j| of the exact contraction — the same order as the fp64 path's
 //     rounding bound (Q24) — and tests/test_gpu_svr.py compares it with the oracle and
 //     with the fp64 k_svr reference (fp32 predictions equal or one ulp apart).
@@ -26,7 +27,7 @@
 // planes of a (tile, chunk) contiguous, so each chunk reaches shared memory by one 1-D bulk copy per
 // operand (cp.async.bulk, the TMA engine) into a 4-stage mbarrier ring.  k_svr_tc: 128 kernels x 64
 // clocks per CTA (M = 128, N = 64, K = 32 per MMA); warp 0 producer, warp 1 TMEM allocation and
-// MMA issue (one elected lane, 36 MMAs per chunk), warps 2-5 epilogue (TMEM lane quarters).  The SV
+// MMA issue (one elected lane, 28 MMAs per chunk), warps 2-5 epilogue (TMEM lane quarters).  The SV
 // range may be split across CTAs (blockIdx.z); each split writes its partial plane P[z], which the
 // finish sums in split order (add_svr_unit), exactly as for k_svr.
 #pragma once
@@ -34,7 +35,7 @@
 
 namespace syn {
 
-constexpr int kTcM = 128, kTcN = 64, kTcKC = 32, kTcDig = 8, kTcStages = 4;
+constexpr int kTcM = 128, kTcN = 64, kTcKC = 32, kTcDig = 7, kTcStages = 4;
 constexpr unsigned kTcAPlane = (unsigned)kTcM * kTcKC, kTcBPlane = (unsigned)kTcN * kTcKC;
 constexpr unsigned kTcABytes = kTcDig * kTcAPlane;   // one 32-SV chunk of U, all digit planes
 constexpr unsigned kTcBBytes = kTcDig * kTcBPlane;   // one chunk of V
@@ -55,29 +56,28 @@ __device__ __forceinline__ unsigned tc_off(int r, int kb) {
     return (unsigned)((r >> 3) * 256 + (kb >> 4) * 128 + (r & 7) * 16 + (kb & 15));
 }
 
-// 16 consecutive values (x[q] in (-1, 1)) -> 8 digit planes, 16 bytes each, at base + p * plane.
-// |x| 2^56 truncated to an integer (exact: the truncation of x to 56 fractional bits) is cut into
-// eight 7-bit magnitude digits from the top, each carrying x's sign: x = sum_p d_p 2^-7(p+1) + r,
-// |d_p| <= 127, |r| < 2^-56 (the same digits as repeated "multiply by 128, truncate").
+// 16 consecutive values (x[q] in (-1, 1)) -> kTcDig digit planes, 16 bytes each, at base + p * plane.
+// X = round(x 2^54) (an integer, |X| < 2^54) is written in balanced base 256, least significant
+// digit first: d = ((X + 128) mod 256) - 128 in [-128, 127], X = (X - d) / 256 (exact), so
+// X = sum_p d_p 256^(kTcDig - 1 - p) with every digit a signed byte; |x - X 2^-54| <= 2^-55.
 __device__ __forceinline__ void tc_store_digits(const double (&x)[16], unsigned char* base, unsigned plane) {
-    unsigned long long m[16];
-    unsigned neg = 0u;
+    long long X[16];
 #pragma unroll
-    for (int q = 0; q < 16; ++q) {
-        m[q] = (unsigned long long)__double2ll_rz(fabs(scalbn(x[q], 56)));   // < 2^56
-        neg |= (x[q] < 0.0 ? 1u : 0u) << q;
-    }
+    for (int q = 0; q < 16; ++q) X[q] = __double2ll_rn(scalbn(x[q], 54));
+    unsigned w[kTcDig][4];
 #pragma unroll
-    for (int p = 0; p < kTcDig; ++p) {
-        unsigned w[4] = {0u, 0u, 0u, 0u};
+    for (int p = kTcDig - 1; p >= 0; --p) {
+        w[p][0] = w[p][1] = w[p][2] = w[p][3] = 0u;
 #pragma unroll
         for (int q = 0; q < 16; ++q) {
-            const int d = (int)((m[q] >> (7 * (kTcDig - 1 - p))) & 127ull);
-            const int sd = ((neg >> q) & 1u) ? -d : d;
-            w[q >> 2] |= ((unsigned)sd & 0xffu) << (8 * (q & 3));
+            const long long d = ((X[q] + 128) & 255) - 128;
+            X[q] = (X[q] - d) >> 8;                                        // exact
+            w[p][q >> 2] |= ((unsigned)d & 0xffu) << (8 * (q & 3));
         }
-        *reinterpret_cast<uint4*>(base + (size_t)p * plane) = make_uint4(w[0], w[1], w[2], w[3]);
     }
+#pragma unroll
+    for (int p = 0; p < kTcDig; ++p)
+        *reinterpret_cast<uint4*>(base + (size_t)p * plane) = make_uint4(w[p][0], w[p][1], w[p][2], w[p][3]);
 }
 
 // U digits for a 128-kernel tile (blockIdx.x, slab-relative) and a 32-SV chunk (blockIdx.y):
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant_
         mbar_init(accb, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (warp == 1) {                                                     // all 512 TMEM columns: 8 x 64
+    if (warp == 1) {                                                     // 512 TMEM columns: 7 x 64 used
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;"
                      :: "r"(svr_su32(tmem_slot)) : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
@@ -254,7 +254,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant_
                       "=r"(v[14]), "=r"(v[15])
                     : "r"(taddr));
                 asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-                const double w = scalbn(1.0, -7 * (L + 2));                        // 2^-7(L+2)
+                const double w = scalbn(1.0, -8 * L - 12);                         // 2^-(8L+12)
 #pragma unroll
                 for (int c = 0; c < 16; ++c) s[c] = __fma_rn((double)(int)v[c], w, s[c]);   // exact products
             }
