@@ -468,25 +468,31 @@ constexpr size_t kTmSlabBytes = 48u << 20;   // D bytes per slab (stays L2-resid
 const DevModel& dm_of(const SweepArgs& a, int m) { return m == 0 ? a.ms : m == 1 ? a.me : a.mx[m - 2]; }
 bool present(const SweepArgs& a, int m) { return m < 2 || a.has_x[m - 2]; }
 
-// k_tm_walk kernels per feature block: a power of two in [32, 256] whose [F + 2][kb] fp32 feature
-// table takes at most 32 KB of shared memory, and no more than the batch needs.
-int tm_kb(int F, long long n_k, long long knob) {
+// k_tm_walk kernels per feature block: a power of two in [32, 1024] whose [F + 2][kb] fp32 feature
+// table fits the budget (64 KB for large batches, 32 KB otherwise), and no more than the batch
+// needs.  Large batches take 1024: a 1024-thread CTA's lanes then cover one tree at a time (the
+// task pools walk unit-major), so the SM's L1 holds one tree (measured: c3 walk 2.54 -> 2.29 ms
+// per slab, c4 0.94 -> 0.89 ms, from 256).
+int tm_kb(int F, long long n_k, long long knob, bool large) {
     const size_t xs = (size_t)(F + 2) * 4;
-    int kb = 256;
-    while (kb > 32 && (xs * kb > 32768 || kb / 2 >= n_k)) kb /= 2;
+    const int kmax = large ? 1024 : n_k >= 2048 ? 512 : 256;   // c5 walk 182 -> 173 us with 512; c2 (1000
+                                                                // kernels, a partial block) 72 -> 87 us
+    const size_t budget = large ? 65536 : 32768;
+    int kb = kmax;
+    while (kb > 32 && (xs * kb > budget || kb / 2 >= n_k)) kb /= 2;
     if (knob > 0) {
         while (kb > 32 && kb > knob) kb /= 2;
-        while (kb < 256 && kb * 2 <= knob) kb *= 2;
+        while (kb < 1024 && kb * 2 <= knob && xs * kb * 2 <= 65536) kb *= 2;
     }
     return kb;
 }
 // k_tm_walk threads per CTA: 1024 (one CTA per SM: one tree window and one feature table per SM
 // instead of two; measured c3 walk 2.62 -> 2.51 ms per slab) for large batches, 512 (two CTAs per
 // SM) when a lane has only a few tasks (c2 72 -> 92 us and c5 181 -> 198 us with 1024)
-int tm_nt(long long slab_tasks, int sms) {
+int tm_nt(long long tasks, int sms) {
     const long long k = knobs().tm_nt.load();
     if (k == 512 || k == 1024) return (int)k;
-    return slab_tasks >= 8LL * 1024 * sms ? 1024 : 512;
+    return tasks >= 8LL * 1024 * sms ? 1024 : 512;
 }
 size_t tm_walk_smem(int F, int kb, int tt, int units, int nt = 1024) {
     return (size_t)tt * sizeof(TmTree) + (size_t)kTmS * nt * 8 + (size_t)kb * (F + 2) * 4 + (size_t)units * 8 +
@@ -509,7 +515,7 @@ bool tm_eligible(const SweepArgs& a, int nm, const DevState* ds) {
         ++nslot;
     }
     if (tt == 0) return false;
-    if (tm_walk_smem(a.F, tm_kb(a.F, a.n_k, knobs().tm_kb.load()), tt, 0) > (size_t)ds->walk_dyn_max) return false;
+    if (tm_walk_smem(a.F, 32, tt, 0, 512) > (size_t)ds->walk_dyn_max) return false;   // the smallest launch
     return tm_finish_smem(nm, 1, a.n_f, (a.F + 2) | 1, nslot) <= (size_t)ds->finish_dyn_max;
 }
 
@@ -556,7 +562,11 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     bool fxall = true;                            // every forest has int32 fixed-point leaves
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0 && !dms[m]->fx32) fxall = false;
-    const int kb = tm_kb(F, n_k, K.tm_kb.load());
+    // large batches (>= 8 tasks per lane): 1024-thread CTAs and 1024-kernel feature blocks
+    int NTW = tm_nt(std::min<long long>(n_k, 1LL << 40) * tt, ds->sms);
+    if (tm_walk_smem(F, 32, tt, 0, NTW) > (size_t)ds->walk_dyn_max) NTW = 512;
+    int kb = tm_kb(F, n_k, K.tm_kb.load(), NTW == 1024);
+    while (kb > 32 && tm_walk_smem(F, kb, tt, 0, NTW) > (size_t)ds->walk_dyn_max) kb /= 2;
     t.kb = kb;
     t.kb_log2 = 0;
     while ((1 << t.kb_log2) < kb) ++t.kb_log2;
@@ -604,7 +614,6 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     int usplit = 0;                               // units of the per-tree split (smode 2)
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0) usplit += dms[m]->units_split;
-    const int NTW = tm_nt((long long)nks * tt, ds->sms);
     const int ctas = (int)std::max<long long>(1, K.tm_ctas.load() > 0 ? K.tm_ctas.load() : (1024LL / NTW) * ds->sms);
     t.s = a;
     int n = 0;
@@ -631,10 +640,10 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         t.nsub = 1;
         const long long lanes = (long long)ctas * NTW;
         while (t.nsub < 8 && (long long)t.nks * tt * t.nsub < lanes && n_f / (2 * t.nsub) >= 8 &&
-               tm_walk_smem(F, kb, tt, 2 * tt * t.nsub) <= (size_t)ds->walk_dyn_max)
+               tm_walk_smem(F, kb, tt, 2 * tt * t.nsub, NTW) <= (size_t)ds->walk_dyn_max)
             t.nsub *= 2;
         if (K.tm_nsub.load() >= 1 && K.tm_nsub.load() <= std::min(n_f, 64) &&
-            tm_walk_smem(F, kb, tt, tt * (int)K.tm_nsub.load()) <= (size_t)ds->walk_dyn_max)
+            tm_walk_smem(F, kb, tt, tt * (int)K.tm_nsub.load(), NTW) <= (size_t)ds->walk_dyn_max)
             t.nsub = (int)K.tm_nsub.load();
         // small batches (2-8 tasks per lane): the longest walks bound the launch's tail, so trees
         // whose expected run count exceeds the model's mean are split into clock sub-ranges
@@ -645,7 +654,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         const long long ksplit = K.tm_split.load();
         const long long per_lane = (long long)t.nks * tt / std::max<long long>(lanes, 1);   // tasks per lane
         if (t.smode == 0 && usplit > tt && (ksplit > 0 || (ksplit < 0 && per_lane >= 2 && per_lane < 8)) &&
-            tm_walk_smem(F, kb, tt, usplit) <= (size_t)ds->walk_dyn_max) {
+            tm_walk_smem(F, kb, tt, usplit, NTW) <= (size_t)ds->walk_dyn_max) {
             t.smode = 2;
             t.units = usplit;
         }

@@ -35,6 +35,7 @@ def _build():
 #   tm_split  per-tree clock sub-range split forced on (trees with many runs cut into pieces)
 #   tm_nosplit  per-tree split off (small batches walk whole trees)
 #   tm_nt1024 k_tm_walk with 1024-thread CTAs (one per SM)
+#   tm_kb1024 1024-thread CTAs with 1024-kernel feature blocks (the large-batch configuration)
 #   tm_nopdl  k_tm_finish launched without programmatic dependent launch
 #   tm_slab   kernel slabs of 64 (several walk + finish launches; finish(i) on the side stream
 #             overlapping walk(i + 1), D double-buffered and re-zeroed by the finishes)
@@ -44,6 +45,7 @@ VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 
             "tm_nsub3": {"tm_nsub": 3}, "tm_nsub64": {"tm_nsub": 64},
             "tm_dyn": {"tm_dyn": 1}, "tm_static": {"tm_dyn": 0}, "tm_nopdl": {"tm_pdl": 0},
             "tm_split": {"tm_split": 1}, "tm_nosplit": {"tm_split": 0}, "tm_nt1024": {"tm_nt": 1024},
+            "tm_kb1024": {"tm_kb": 1024, "tm_nt": 1024},
             "tm_slab": {"tm_slab": 64, "tm_kb": 32},
             "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0}}
 KNOB_DEFAULTS = {"algo": 0, "tm_kb": 0, "tm_ctas": 0, "tm_nsub": 0, "tm_split": -1, "tm_dyn": -1, "tm_pdl": 1,
