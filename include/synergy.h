@@ -39,9 +39,10 @@
  *     captured returns SYN_ERR_UNSUPPORTED instead.
  *   - Paths: the tree-major kernels (k_tm_walk + k_tm_finish) when every forest's leaves fit the
  *     int64 fixed-point range and the per-tree task table fits shared memory (about 25 000 trees
- *     per call, any F); otherwise the general exact kernels (k_gen_forest + k_gen_finish: direct
- *     traversal, 320-bit exact leaf sums), which accept every valid model.  Both return the same
- *     bits.
+ *     per call, any F), or for small batches (at most one kernel per SM) the single-launch
+ *     k_tm_small (direct walks and the finish in one CTA per kernel); otherwise the general exact
+ *     kernels (k_gen_forest + k_gen_finish: direct traversal, 320-bit exact leaf sums), which
+ *     accept every valid model.  All return the same bits.
  *   - Layouts are row-major and contiguous: features [n_kernels][n_features] fp32,
  *     predictions [n_kernels][n_freqs] fp32, choices [n_kernels][n_targets] int32.
  *   - Handles (models, clock tables, workspaces) are bound to the device they were created
@@ -277,8 +278,12 @@ syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms
 /* Tuning knobs (launch-configuration choices only; results are identical for every setting), for
  * tests and benchmarks.  Initialised once from the environment (SYNERGY_<KEY upper-case>), then
  * process-wide.  Keys: "algo" (0 automatic, 1 force the general exact kernels), "tm_kb" (k_tm_walk
- * kernels per feature block, 32..256), "tm_ctas", "tm_nsub", "tm_dyn" (-1 automatic), "tm_pdl",
- * "tm_slab", "tm_pipe", "tm_kt", "tm_split" (-1 automatic), "gen_kt", "svr_splits"; 0 = automatic
+ * kernels per feature block, 32..1024), "tm_nt" (k_tm_walk threads per CTA, 512 or 1024), "tm_ctas",
+ * "tm_nsub", "tm_split" (per-tree clock-range split, -1 automatic, 0 off, 1 on), "split_piece"
+ * (model create: target cost of one split piece in quarters of the mean tree cost, default 4),
+ * "tm_dyn" (task pools, -1 automatic), "tm_pdl" (default 1), "tm_slab", "tm_pipe" (default 1),
+ * "tm_kt", "gen_kt", "svr_splits", "svr_tc" (tcgen05 SVR contraction, default 1), "tm_small"
+ * (single-launch k_tm_small for small batches: -1 automatic, 0 off, 1 on); 0 = automatic
  * unless noted.  INVALID_ARG: unknown key. */
 syn_status synergy_config_set(const char *key, int64_t value);
 syn_status synergy_config_get(const char *key, int64_t *value);

@@ -110,7 +110,7 @@ struct SweepArgs {
     int def;                 // default clock index; -1 = raw (predict only)
     int n_t;
     int kind[kMaxTargets];
-    float x[kMaxTargets];
+    double frac[kMaxTargets];  // x / 100 (fp64, host: the oracle's division)
     int* choice;             // [n_k][n_t] (sweep)
     float* S_out;            // [n_k][n_f] or null
     float* E_out;
@@ -128,7 +128,7 @@ struct SelectArgs {
     int def;
     int n_t;
     int kind[kMaxTargets];
-    float x[kMaxTargets];
+    double frac[kMaxTargets];  // x / 100 (fp64, host: the oracle's division)
     int* choice;
 };
 

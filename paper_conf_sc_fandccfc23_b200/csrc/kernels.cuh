@@ -3,15 +3,15 @@
 //   combine()        a model's raw output from its exact forest sum: linear member, forest mean
 //                    (Q7/Q8)
 //   finish_tile4()   SVR member, default-clock normalisation (L69), then per target the objective /
-//                    constraint and the masked lowest-index argmin (L253-L271, L322) with warp
-//                    shuffles; used by k_tm_finish and k_gen_finish
+//                    constraint and the masked lowest-index argmin (L253-L271, L322) on integer
+//                    keys with warp min-reductions; used by k_tm_finish and k_gen_finish
 //   k_select         standalone selection over predictions in HBM (one warp per kernel)
 //   k_pareto, k_choice_error, k_error_reduce, k_plan   NEXT f3 / f4 (Pareto front, choice error,
 //                    plan emission)
 //
 // Arithmetic contract (Q15): the oracle's op sequence — fp64 fma chain for the linear
 // member, exact leaf sum rounded once then / T, fp64 normalisation rounded once to fp32, fp64
-// keys / thresholds; every fp64 op is an explicit _rn intrinsic and the library is built with
+// thresholds (compared exactly on the floats, see select_target); every fp64 op is an explicit _rn intrinsic and the library is built with
 // --fmad=false, so nothing is contracted.  Ties: lexicographic (key, index) minimum.
 #pragma once
 #include "device_util.cuh"
@@ -22,15 +22,6 @@ namespace syn {
 __device__ __forceinline__ bool valid_pred(float s, float e) {
     // DESIGN.md Q16: finite and strictly positive speedup and energy
     return isfinite(s) && isfinite(e) && s > 0.0f && e > 0.0f;
-}
-
-__device__ __forceinline__ void argmin_shfl(double& key, int& idx) {
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) {
-        const double ok = __shfl_xor_sync(0xffffffffu, key, off);
-        const int oi = __shfl_xor_sync(0xffffffffu, idx, off);
-        if (ok < key || (ok == key && oi < idx)) { key = ok; idx = oi; }
-    }
 }
 
 // Model output from its forest sum (the exact leaf sum rounded once to fp64; oracle order: linear
@@ -50,80 +41,114 @@ __device__ __forceinline__ double combine(const DevModel& m, double forest_sum, 
     return out;
 }
 
-// Selection baselines of one row (Q14-Q16): returns false if the default clock's
-// prediction is invalid (every target then -1); else E_def, S_def and the minimum-energy point's
-// E_min, S_minE (lowest index among equal minima, L265).  Whole warp, result in every lane.
+// Selection on integer keys.  A valid prediction (Q16) is a positive finite float, and the bit
+// patterns of positive finite floats and doubles order like their values; every key below is
+// such a value or (MAX_PERF, ES) the complement of one.  So a target's masked lexicographic
+// (key, index) minimum is a lane-local strict-< scan in clock order followed by warp
+// min-reductions (REDUX): first over the key words, then over the indices of the lanes that hold
+// the minimum.  An invalid or infeasible clock has the all-ones key, which no valid key reaches.
+__device__ __forceinline__ bool valid_bits(unsigned b) { return b - 1u < 0x7f7fffffu; }   // (0, FLT_MAX]
+
+__device__ __forceinline__ int warp_argmin32(unsigned key, unsigned idx) {
+    const unsigned m = __reduce_min_sync(0xffffffffu, key);
+    const unsigned i = __reduce_min_sync(0xffffffffu, key == m ? idx : 0xffffffffu);
+    return m == 0xffffffffu ? -1 : (int)i;
+}
+
+__device__ __forceinline__ int warp_argmin64(unsigned long long key, unsigned idx) {
+    const unsigned hi = (unsigned)(key >> 32), lo = (unsigned)key;
+    const unsigned mh = __reduce_min_sync(0xffffffffu, hi);
+    const unsigned ml = __reduce_min_sync(0xffffffffu, hi == mh ? lo : 0xffffffffu);
+    const unsigned i = __reduce_min_sync(0xffffffffu, (hi == mh && lo == ml) ? idx : 0xffffffffu);
+    return (mh == 0xffffffffu && ml == 0xffffffffu) ? -1 : (int)i;
+}
+
+struct RowBase {
+    double E_def, S_def, E_min, S_minE;
+};
+
+// Selection baselines of one row (Q14-Q16): false if the default clock's prediction is
+// invalid (every target then -1); else E_def, S_def and the minimum-energy point's E_min, S_minE
+// (lowest index among equal minima, L265).  Whole warp, result in every lane.
 __device__ __forceinline__ bool select_baseline(const float* S, const float* E, int n_f, int def, int lane,
-                                                double& E_def, double& S_def, double& E_min, double& S_minE) {
+                                                RowBase& b) {
     const float sd = S[def], ed = E[def];
-    if (!valid_pred(sd, ed)) return false;
-    double be = CUDART_INF;
-    int bi = INT_MAX;
+    if (!(valid_bits(__float_as_uint(sd)) && valid_bits(__float_as_uint(ed)))) return false;
+    unsigned bk = 0xffffffffu, bi = 0xffffffffu;
     for (int i = lane; i < n_f; i += 32) {
-        const float s = S[i], e = E[i];
-        if (valid_pred(s, e) && (double)e < be) { be = (double)e; bi = i; }
+        const unsigned su = __float_as_uint(S[i]), eu = __float_as_uint(E[i]);
+        const unsigned k = (valid_bits(su) && valid_bits(eu)) ? eu : 0xffffffffu;
+        if (k < bk) { bk = k; bi = i; }
     }
-    argmin_shfl(be, bi);
-    E_def = (double)ed;
-    S_def = (double)sd;
-    E_min = (double)E[bi];
-    S_minE = (double)S[bi];
+    const int im = warp_argmin32(bk, bi);                          // >= 0: the default is valid
+    b.E_def = (double)ed;
+    b.S_def = (double)sd;
+    b.E_min = (double)E[im];
+    b.S_minE = (double)S[im];
     return true;
 }
 
 // One target of one row: the lowest index minimising the target's key
-// among valid feasible clocks, -1 if none.  P2/P3: direct EDP / ED2P predictions or null.
+// among valid feasible clocks, -1 if none.  frac = x / 100 in fp64 (host-computed, the oracle's
+// division).  P2/P3: direct EDP / ED2P predictions or null.  A constraint (double)e <= thr holds
+// for a float e iff e <= RD_float(thr) (the largest float not above thr), and (double)s >= thr
+// iff s >= RU_float(thr), so the feasibility tests run on the floats.
 __device__ __forceinline__ int select_target(const float* S, const float* E, const float* P2, const float* P3,
-                                             int n_f, int kd, float x, double E_def, double S_def,
-                                             double E_min, double S_minE, int lane) {
-    const double frac = __ddiv_rn((double)x, 100.0);
-    const double thr_es = __dsub_rn(E_def, __dmul_rn(frac, __dsub_rn(E_def, E_min)));
-    const double thr_pl = __dsub_rn(S_def, __dmul_rn(frac, __dsub_rn(S_def, S_minE)));
-    // absolute-saving reading (L11/L46, Q1): E <= (1 - x%) E_def, S >= (1 - x%) S_def
-    const double thr_es_abs = __dmul_rn(__dsub_rn(1.0, frac), E_def);
-    const double thr_pl_abs = __dmul_rn(__dsub_rn(1.0, frac), S_def);
-    double bk = CUDART_INF;
-    int bx = INT_MAX;
+                                             int n_f, int kd, double frac, const RowBase& b, int lane) {
+    if (kd == 2 || kd == 3) {                                       // MIN_EDP e*t, MIN_ED2P e*t^2
+        const float* P = kd == 2 ? P2 : P3;
+        unsigned long long bk = ~0ull;
+        unsigned bi = 0xffffffffu;
+        for (int i = lane; i < n_f; i += 32) {
+            const float sf = S[i], ef = E[i];
+            if (!(valid_bits(__float_as_uint(sf)) && valid_bits(__float_as_uint(ef)))) continue;
+            unsigned long long k;
+            if (P) {                                                // direct prediction, valid too
+                const unsigned pu = __float_as_uint(P[i]);
+                if (!valid_bits(pu)) continue;
+                k = pu;
+            } else {                                                // e / s (/ s): positive finite
+                double q = __ddiv_rn((double)ef, (double)sf);
+                if (kd == 3) q = __ddiv_rn(q, (double)sf);
+                k = (unsigned long long)__double_as_longlong(q);
+            }
+            if (k < bk) { bk = k; bi = i; }
+        }
+        return warp_argmin64(bk, bi);
+    }
+    float ebound = CUDART_INF_F, sbound = -CUDART_INF_F;            // feasible: e <= ebound, s >= sbound
+    if (kd == 4)                                                    // ES_x: E <= E_def - x% (E_def - E_min)
+        ebound = __double2float_rd(__dsub_rn(b.E_def, __dmul_rn(frac, __dsub_rn(b.E_def, b.E_min))));
+    else if (kd == 5)                                               // PL_x: S >= S_def - x% (S_def - S_minE)
+        sbound = __double2float_ru(__dsub_rn(b.S_def, __dmul_rn(frac, __dsub_rn(b.S_def, b.S_minE))));
+    else if (kd == 6)                                               // ES_ABS_x (L11/L46, Q1): E <= (1 - x%) E_def
+        ebound = __double2float_rd(__dmul_rn(__dsub_rn(1.0, frac), b.E_def));
+    else if (kd == 7)                                               // PL_ABS_x: S >= (1 - x%) S_def
+        sbound = __double2float_ru(__dmul_rn(__dsub_rn(1.0, frac), b.S_def));
+    const bool max_s = kd == 0 || kd == 4 || kd == 6;               // key -s: complement of s's bits
+    unsigned bk = 0xffffffffu, bi = 0xffffffffu;
     for (int i = lane; i < n_f; i += 32) {
         const float sf = S[i], ef = E[i];
-        if (!valid_pred(sf, ef)) continue;
-        const double s = (double)sf, e = (double)ef;
-        double key;
-        bool feas = true;
-        switch (kd) {
-            case 0: key = -s; break;                                   // MAX_PERF
-            case 1: key = e; break;                                    // MIN_ENERGY
-            case 2:                                                    // MIN_EDP  e*t
-                if (P2) { const float p = P2[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
-                else key = __ddiv_rn(e, s);
-                break;
-            case 3:                                                    // MIN_ED2P e*t^2
-                if (P3) { const float p = P3[i]; feas = isfinite(p) && p > 0.0f; key = (double)p; }
-                else key = __ddiv_rn(__ddiv_rn(e, s), s);
-                break;
-            case 4: feas = (e <= thr_es); key = -s; break;             // ES_x
-            case 5: feas = (s >= thr_pl); key = e; break;              // PL_x
-            case 6: feas = (e <= thr_es_abs); key = -s; break;         // ES_ABS_x
-            default: feas = (s >= thr_pl_abs); key = e; break;         // PL_ABS_x
-        }
-        if (feas && (key < bk || (key == bk && i < bx))) { bk = key; bx = i; }
+        const unsigned su = __float_as_uint(sf), eu = __float_as_uint(ef);
+        const bool ok = valid_bits(su) && valid_bits(eu) && ef <= ebound && sf >= sbound;
+        const unsigned k = ok ? (max_s ? ~su : eu) : 0xffffffffu;
+        if (k < bk) { bk = k; bi = i; }
     }
-    argmin_shfl(bk, bx);
-    return bx == INT_MAX ? -1 : bx;
+    return warp_argmin32(bk, bi);
 }
 
 // Every target of one row, one warp (standalone selection and the choice-error truth).
 __device__ __forceinline__ void select_row_warp(const float* S, const float* E, const float* P2,
                                                 const float* P3, int n_f, int def,
-                                                int n_t, const int* kind, const float* xs,
+                                                int n_t, const int* kind, const double* frac,
                                                 int* out, int lane) {
-    double E_def, S_def, E_min, S_minE;
-    if (!select_baseline(S, E, n_f, def, lane, E_def, S_def, E_min, S_minE)) {
+    RowBase b;
+    if (!select_baseline(S, E, n_f, def, lane, b)) {
         for (int t = lane; t < n_t; t += 32) out[t] = -1;
         return;
     }
     for (int t = 0; t < n_t; ++t) {
-        const int c = select_target(S, E, P2, P3, n_f, kind[t], xs[t], E_def, S_def, E_min, S_minE, lane);
+        const int c = select_target(S, E, P2, P3, n_f, kind[t], frac[t], b, lane);
         if (lane == 0) out[t] = c;
     }
 }
@@ -175,20 +200,20 @@ __device__ __forceinline__ void finish_tile4(const SweepArgs& a, double* const* 
     const int tb = (threadIdx.x >> 5) * per, te = min(ntask, tb + per);
     int row = -1;
     bool base_ok = false;
-    double E_def = 0.0, S_def = 0.0, E_min = 0.0, S_minE = 0.0;
+    RowBase base{};
     for (int task = tb; task < te; ++task) {
         const int kl = task / n_t, t = task - kl * n_t;
         const float* S = sv[0] + (size_t)kl * n_f;
         const float* E = sv[1] + (size_t)kl * n_f;
         if (kl != row) {
             row = kl;
-            base_ok = select_baseline(S, E, n_f, a.def, lane, E_def, S_def, E_min, S_minE);
+            base_ok = select_baseline(S, E, n_f, a.def, lane, base);
         }
         int c = -1;
         if (base_ok)
             c = select_target(S, E, mv[2] ? sv[2] + (size_t)kl * n_f : nullptr,
-                              mv[3] ? sv[3] + (size_t)kl * n_f : nullptr, n_f, a.kind[t], a.x[t],
-                              E_def, S_def, E_min, S_minE, lane);
+                              mv[3] ? sv[3] + (size_t)kl * n_f : nullptr, n_f, a.kind[t], a.frac[t], base,
+                              lane);
         if (lane == 0) a.choice[(k0 + kl) * n_t + t] = c;
     }
 }
@@ -199,7 +224,7 @@ __global__ void __launch_bounds__(256) k_select(const __grid_constant__ SelectAr
     const int lane = threadIdx.x & 31;
     const long long warps = (long long)gridDim.x * (blockDim.x >> 5);
     for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < a.n_k; k += warps) {
-        select_row_warp(a.S + k * a.n_f, a.E + k * a.n_f, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.x,
+        select_row_warp(a.S + k * a.n_f, a.E + k * a.n_f, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.frac,
                         a.choice + k * a.n_t, lane);
     }
 }
@@ -246,7 +271,7 @@ __global__ void __launch_bounds__(256) k_choice_error(const __grid_constant__ Se
     for (long long k = (long long)blockIdx.x * (blockDim.x >> 5) + w; k < a.n_k; k += warps) {
         const float* s = a.S + k * a.n_f;
         const float* e = a.E + k * a.n_f;
-        select_row_warp(s, e, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.x, truth[w], lane);
+        select_row_warp(s, e, nullptr, nullptr, a.n_f, a.def, a.n_t, a.kind, a.frac, truth[w], lane);
         __syncwarp();
         if (lane < a.n_t) {
             const int ip = __ldg(pred + k * a.n_t + lane), it = truth[w][lane];

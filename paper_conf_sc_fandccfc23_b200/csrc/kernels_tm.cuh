@@ -388,72 +388,71 @@ __global__ void __launch_bounds__(256) k_cut_blocks(const uint4* __restrict__ in
     out[2 * b + 1] = make_uint4(g[0], g[1], g[2], g[3]);
 }
 
-// Finish of KT kernels per CTA: exact prefix sums of the D rows (zeroing them), forest mean,
-// linear member, then finish_tile4 (SVR members, normalisation, selection).
-__global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArgs t) {
+// Shared-memory layout of a finish tile of KT kernels: fp64 and fp32 outputs per (model, kernel,
+// clock), the clock table, the kernels' features (stride XS) and the exact sums [KT][nslot][n_f].
+struct TmFinishSmem {
+    double* mv0;     // [NM][KT][n_f]
+    float* sv0;      // [NM][KT][n_f]
+    float* fr;       // [n_f]
+    float* xk;       // [KT][XS]
+    long long* sD;   // [KT][nslot][n_f], 16-byte aligned
+};
+__device__ __forceinline__ TmFinishSmem tm_finish_layout(unsigned char* smem, int NM, int KT, int n_f, int XS) {
+    TmFinishSmem L;
+    L.mv0 = reinterpret_cast<double*>(smem);
+    L.sv0 = reinterpret_cast<float*>(L.mv0 + (size_t)NM * KT * n_f);
+    L.fr = L.sv0 + (size_t)NM * KT * n_f;
+    L.xk = L.fr + n_f;
+    L.sD = reinterpret_cast<long long*>(L.xk + KT * XS + 1);
+    L.sD = reinterpret_cast<long long*>((reinterpret_cast<uintptr_t>(L.sD) + 15) & ~(uintptr_t)15);
+    return L;
+}
+
+// The finish of nk kernels (k0 = global index of the first) whose exact leaf sums per (kernel,
+// slot, clock) sit in L.sD: as difference arrays (scan: exact prefix sums first, in place) or as
+// the sums themselves.  Forest mean and linear member per (model, clock) (combine), then
+// finish_tile4 (SVR members, normalisation, selection).  Whole CTA; the caller has synchronised.
+__device__ __forceinline__ void tm_finish_tile(const TmArgs& t, const TmFinishSmem& L, int KT, int nk, long long k0,
+                                               bool scan) {
     const SweepArgs& a = t.s;
-    extern __shared__ __align__(16) unsigned char smem[];
-    const int n_f = a.n_f, F = a.F, KT = a.tile_k, XS = a.xs, NM = t.nm;
-    const int k0s = blockIdx.x * KT;
-    const int nk = min(KT, t.nks - k0s);
-    const long long k0 = t.slab0 + k0s;
-    double* mv0 = reinterpret_cast<double*>(smem);                            // [NM][KT][n_f]
-    float* sv0 = reinterpret_cast<float*>(mv0 + (size_t)NM * KT * n_f);       // [NM][KT][n_f]
-    float* fr = sv0 + (size_t)NM * KT * n_f;
-    float* xk = fr + n_f;                                                     // [KT][XS]
-    long long* sD = reinterpret_cast<long long*>(xk + KT * XS + 1);           // [KT][nslot][n_f]
-    sD = reinterpret_cast<long long*>((reinterpret_cast<uintptr_t>(sD) + 15) & ~(uintptr_t)15);
-    const float* gfeat = a.features + k0 * F;
-    for (int e = threadIdx.x; e < nk * F; e += blockDim.x) {
-        const int r = e / F;
-        xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
-    }
-    for (int i = threadIdx.x; i < n_f; i += blockDim.x) fr[i] = __ldg(a.freqs + i);
-    // launched as a programmatic dependent of k_tm_walk (same stream): everything above overlaps
-    // the walk's tail; D is read only after the walk grid has completed (no-op otherwise)
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    // this CTA's D rows are one contiguous region: stage it with independent coalesced loads,
-    // then zero it for the next call
-    long long* gD = t.D + (size_t)k0s * t.nslot * n_f;
-    const int nd = nk * t.nslot * n_f;
-    for (int e = threadIdx.x; e < nd; e += blockDim.x) sD[e] = __ldcg(gD + e);
-    __syncthreads();
-    for (int e = threadIdx.x; e < nd; e += blockDim.x) gD[e] = 0;
+    const int n_f = a.n_f, F = a.F, XS = a.xs, NM = t.nm;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     for (int p = warp; p < NM * nk; p += nw) {                                // p = kernel * NM + model
         const int pk = p / NM, pm = p - pk * NM;
         if (pm >= 2 && !a.has_x[pm - 2]) continue;
         const DevModel& m = model_of(a, pm);
-        double* out = mv0 + ((size_t)pm * KT + pk) * n_f;
-        const float* xrow = xk + pk * XS;
+        double* out = L.mv0 + ((size_t)pm * KT + pk) * n_f;
+        const float* xrow = L.xk + pk * XS;
         const int slot = t.slot_of[pm];
         if (slot < 0) {
-            for (int i = lane; i < n_f; i += 32) out[i] = combine(m, 0.0, xrow, fr[i], F);
+            for (int i = lane; i < n_f; i += 32) out[i] = combine(m, 0.0, xrow, L.fr[i], F);
             continue;
         }
-        long long* Dm = sD + ((size_t)pk * t.nslot + slot) * n_f;
-        const int chunk = (n_f + 31) / 32;
-        const int i0 = min(n_f, lane * chunk), i1 = min(n_f, i0 + chunk);
-        long long run = 0;
-        for (int i = i0; i < i1; ++i) run += Dm[i];
-        long long excl = run;                                                 // inclusive scan of chunk sums
+        long long* Dm = L.sD + ((size_t)pk * t.nslot + slot) * n_f;
+        if (scan) {
+            const int chunk = (n_f + 31) / 32;
+            const int i0 = min(n_f, lane * chunk), i1 = min(n_f, i0 + chunk);
+            long long run = 0;
+            for (int i = i0; i < i1; ++i) run += Dm[i];
+            long long excl = run;                                             // inclusive scan of chunk sums
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const long long y = __shfl_up_sync(0xffffffffu, excl, off);
-            if (lane >= off) excl += y;
+            for (int off = 1; off < 32; off <<= 1) {
+                const long long y = __shfl_up_sync(0xffffffffu, excl, off);
+                if (lane >= off) excl += y;
+            }
+            excl -= run;
+            for (int i = i0; i < i1; ++i) {                                   // exact prefix sums in place
+                excl += Dm[i];
+                Dm[i] = excl;
+            }
+            __syncwarp();
         }
-        excl -= run;
-        for (int i = i0; i < i1; ++i) {                                       // exact prefix sums in place
-            excl += Dm[i];
-            Dm[i] = excl;
-        }
-        __syncwarp();
         // every clock independently (lane-strided, unrolled: the fp64 chains overlap)
         const double inv = m.fx_inv;
 #pragma unroll 4
         for (int i = lane; i < n_f; i += 32) {
             const double forest_sum = __dmul_rn(__ll2double_rn(Dm[i]), inv);  // RN(exact sum)
-            out[i] = combine(m, forest_sum, xrow, fr[i], F);
+            out[i] = combine(m, forest_sum, xrow, L.fr[i], F);
         }
     }
     __syncthreads();
@@ -461,10 +460,125 @@ __global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArg
     float* sv[4];
     for (int m = 0; m < 4; ++m) {
         const bool present = m < 2 || (NM > 2 && a.has_x[m - 2]);
-        mv[m] = present ? mv0 + (size_t)m * KT * n_f : nullptr;
-        sv[m] = present ? sv0 + (size_t)m * KT * n_f : nullptr;
+        mv[m] = present ? L.mv0 + (size_t)m * KT * n_f : nullptr;
+        sv[m] = present ? L.sv0 + (size_t)m * KT * n_f : nullptr;
     }
     finish_tile4(a, mv, sv, nk, k0);
+}
+
+// Finish of KT kernels per CTA after k_tm_walk: stage and zero the D rows, exact prefix sums,
+// then tm_finish_tile.
+__global__ void __launch_bounds__(256) k_tm_finish(const __grid_constant__ TmArgs t) {
+    const SweepArgs& a = t.s;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int n_f = a.n_f, F = a.F, KT = a.tile_k, XS = a.xs;
+    const int k0s = blockIdx.x * KT;
+    const int nk = min(KT, t.nks - k0s);
+    const long long k0 = t.slab0 + k0s;
+    const TmFinishSmem L = tm_finish_layout(smem, t.nm, KT, n_f, XS);
+    const float* gfeat = a.features + k0 * F;
+    for (int e = threadIdx.x; e < nk * F; e += blockDim.x) {
+        const int r = e / F;
+        L.xk[r * XS + (e - r * F)] = __ldg(gfeat + e);
+    }
+    for (int i = threadIdx.x; i < n_f; i += blockDim.x) L.fr[i] = __ldg(a.freqs + i);
+    // launched as a programmatic dependent of k_tm_walk (same stream): everything above overlaps
+    // the walk's tail; D is read only after the walk grid has completed (no-op otherwise)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    // this CTA's D rows are one contiguous region: stage it with independent coalesced loads,
+    // then zero it for the next call
+    long long* gD = t.D + (size_t)k0s * t.nslot * n_f;
+    const int nd = nk * t.nslot * n_f;
+    for (int e = threadIdx.x; e < nd; e += blockDim.x) L.sD[e] = __ldcg(gD + e);
+    __syncthreads();
+    for (int e = threadIdx.x; e < nd; e += blockDim.x) gD[e] = 0;
+    tm_finish_tile(t, L, KT, nk, k0, true);
+}
+
+// Single-launch path for small batches: one CTA per kernel walks every (tree,
+// clock) pair directly from the root on the clock-cut blocks (clock i enters as i + 0.5, as in
+// k_tm_walk), adds the leaf's exact fixed-point value into the kernel's int64 sums in shared
+// memory (order-free), then runs the finish in the same CTA: no difference arrays, no second
+// launch.  STAGE: the call's clock-cut blocks fit in shared memory and are copied there first
+// (coalesced 16-byte loads, all independent), so the walks' dependent block fetches cost shared-
+// memory latency instead of L2 / DRAM latency.
+template <bool FXALL, bool STAGE>
+__global__ void __launch_bounds__(512, 1) k_tm_small(const __grid_constant__ TmArgs t) {
+    const SweepArgs& a = t.s;
+    extern __shared__ __align__(16) unsigned char smem[];
+    const int n_f = a.n_f, F = a.F, XS = a.xs;
+    const long long k0 = t.slab0 + blockIdx.x;
+    const TmFinishSmem L = tm_finish_layout(smem, t.nm, 1, n_f, XS);
+    float* xw = reinterpret_cast<float*>(L.sD + (size_t)t.nslot * n_f);      // [F + 2] walk features
+    uint4* sblk = reinterpret_cast<uint4*>((reinterpret_cast<uintptr_t>(xw + F + 2) + 15) & ~(uintptr_t)15);
+    __shared__ int s_fx[4];
+    __shared__ double s_scale[4];
+    __shared__ const uint4* s_blocks[4];                                      // per model: its blocks
+    const int T0 = trees_of(a, 0), T1 = trees_of(a, 1), T2 = t.nm > 2 ? trees_of(a, 2) : 0;
+    const int c1 = T0, c2 = c1 + T1, c3 = c2 + T2, TT = c3 + (t.nm > 2 ? trees_of(a, 3) : 0);
+    if (threadIdx.x == 0) {
+        size_t off = 0;                                                       // staged: uint4 offset
+        for (int m = 0; m < 4; ++m) {
+            if (!trees_of(a, m)) continue;
+            const DevModel& d = model_of(a, m);
+            s_fx[m] = d.fx32;
+            s_scale[m] = d.fx_scale;
+            s_blocks[m] = STAGE ? sblk + off : d.blocks;
+            off += 2 * (size_t)d.nblk;
+        }
+    }
+    if (STAGE) {                                                              // every model's blocks, in order
+        size_t off = 0;
+        for (int m = 0; m < 4; ++m) {
+            if (!trees_of(a, m)) continue;
+            const DevModel& d = model_of(a, m);
+            const int n16 = 2 * d.nblk;
+            for (int e = threadIdx.x; e < n16; e += blockDim.x) sblk[off + e] = __ldg(d.blocks + e);
+            off += n16;
+        }
+    }
+    const float* gfeat = a.features + k0 * F;
+    for (int e = threadIdx.x; e < F; e += blockDim.x) {
+        const float v = __ldg(gfeat + e);
+        L.xk[e] = v;
+        xw[e] = v;
+    }
+    if (threadIdx.x < 2) xw[F + threadIdx.x] = 0.0f;                          // row F unused, F + 1 = 0
+    for (int i = threadIdx.x; i < n_f; i += blockDim.x) L.fr[i] = __ldg(a.freqs + i);
+    for (int e = threadIdx.x; e < t.nslot * n_f; e += blockDim.x) L.sD[e] = 0;
+    __syncthreads();
+    const unsigned xs_a = su32(xw);
+    const int nw = TT * n_f;
+    for (int w = threadIdx.x; w < nw; w += blockDim.x) {
+        const int tree = w / n_f, i = w - tree * n_f;
+        const int mi = tree < c1 ? 0 : tree < c2 ? 1 : tree < c3 ? 2 : 3;
+        const DevModel& d = model_of(a, mi);
+        const uint4* blocks = s_blocks[mi];
+        int bk = __ldg(d.broot + (tree - (mi == 0 ? 0 : mi == 1 ? c1 : mi == 2 ? c2 : c3)));
+        const float clk = (float)i + 0.5f;
+        while (true) {
+            uint4 A, B;
+            if (STAGE) {
+                A = blocks[2 * (size_t)bk];
+                B = blocks[2 * (size_t)bk + 1];
+            } else {
+                ldg_blk256(blocks + 2 * (size_t)bk, A, B);
+            }
+            float cb;
+            bool at_leaf;
+            const unsigned g = tm_step(A, B, xs_a, 4u, clk, cb, at_leaf);
+            if (at_leaf) {
+                const long long v = (FXALL || s_fx[mi]) ? (long long)(int)g
+                                                        : __double2ll_rn(__dmul_rn((double)__uint_as_float(g), s_scale[mi]));
+                atomicAdd(reinterpret_cast<unsigned long long*>(L.sD + (size_t)t.slot_of[mi] * n_f + i),
+                          (unsigned long long)v);
+                break;
+            }
+            bk = (int)g;
+        }
+    }
+    __syncthreads();
+    tm_finish_tile(t, L, 1, 1, k0, false);
 }
 
 }  // namespace syn

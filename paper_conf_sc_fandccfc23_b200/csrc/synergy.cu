@@ -171,8 +171,8 @@ bool current_device_is(int dev) {
 // at run time (tests use it to force launch-configuration variants).  0 / -1 = automatic.
 struct Knobs {
     std::atomic<long long> algo{0};       // 0 auto, 1 force k_gen (general exact path)
-    std::atomic<long long> tm_kb{0};      // k_tm_walk kernels per feature block (32..256)
-    std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default 2 per SM)
+    std::atomic<long long> tm_kb{0};      // k_tm_walk kernels per feature block (32..1024)
+    std::atomic<long long> tm_ctas{0};    // k_tm_walk CTAs (default one wave: 1024 / threads-per-CTA per SM)
     std::atomic<long long> tm_nsub{0};    // clock sub-ranges per (kernel, tree) task
     std::atomic<long long> tm_split{-1};  // per-tree sub-range split: -1 auto (small batches), 0 off, 1 on
     std::atomic<long long> tm_nt{0};      // k_tm_walk threads per CTA: 0 automatic, 512 or 1024
@@ -185,6 +185,7 @@ struct Knobs {
     std::atomic<long long> gen_kt{0};     // k_gen_finish kernels per CTA
     std::atomic<long long> svr_splits{0}; // k_svr / k_svr_tc SV-range splits (0: fill the SMs)
     std::atomic<long long> svr_tc{1};     // SVR contraction on tcgen05 (int8 digit products); 0: fp64 k_svr
+    std::atomic<long long> tm_small{-1};  // single-launch k_tm_small: -1 auto (small batches), 0 off, 1 on
 };
 Knobs g_knobs;
 struct KnobName {
@@ -195,7 +196,7 @@ const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_
                            {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_nt", &g_knobs.tm_nt}, {"split_piece", &g_knobs.split_piece}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
                            {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
                            {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits},
-                           {"svr_tc", &g_knobs.svr_tc}};
+                           {"svr_tc", &g_knobs.svr_tc}, {"tm_small", &g_knobs.tm_small}};
 std::once_flag g_knobs_once;
 
 const Knobs& knobs() {
@@ -217,6 +218,7 @@ struct DevState {
     int optin = 227 * 1024;               // max shared memory per CTA (opt-in)
     int walk_dyn_max = 0;                 // dynamic shared memory k_tm_walk / k_tm_finish may take
     int finish_dyn_max = 0;
+    int small_dyn_max = 0;                // k_tm_small
     cudaError_t init_err = cudaSuccess;
     cudaMemPool_t pool = nullptr;         // library-owned stream-ordered pool (release threshold max)
     std::mutex occ_mu;
@@ -255,6 +257,10 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_tm_walk<1024, true, true>, d.optin));
         chk(allow_smem(k_tm_walk<1024, false, true>, d.optin));
         chk(allow_smem(k_tm_finish, d.optin));
+        chk(allow_smem(k_tm_small<true, false>, d.optin));
+        chk(allow_smem(k_tm_small<false, false>, d.optin));
+        chk(allow_smem(k_tm_small<true, true>, d.optin));
+        chk(allow_smem(k_tm_small<false, true>, d.optin));
         chk(allow_smem(k_svr<1>, d.optin));
         chk(allow_smem(k_svr<2>, d.optin));
         chk(allow_smem(k_svr<3>, d.optin));
@@ -271,6 +277,8 @@ DevState* dev_state(int dev) {
         d.walk_dyn_max = d.optin - (int)fa.sharedSizeBytes;
         if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_finish));
         d.finish_dyn_max = d.optin - (int)fa.sharedSizeBytes;
+        if (e == cudaSuccess) chk(cudaFuncGetAttributes(&fa, k_tm_small<false, true>));
+        d.small_dyn_max = d.optin - (int)fa.sharedSizeBytes;
         cudaMemPoolProps props;
         memset(&props, 0, sizeof props);
         props.allocType = cudaMemAllocationTypePinned;
@@ -562,6 +570,43 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     bool fxall = true;                            // every forest has int32 fixed-point leaves
     for (int m = 0; m < nm; ++m)
         if (t.slot_of[m] >= 0 && !dms[m]->fx32) fxall = false;
+    a.xs = (F + 2) | 1;
+    // small batches (at most one kernel per SM, at most 4096 (tree, clock) walks per kernel): one
+    // launch, k_tm_small, one CTA per kernel with direct walks and the finish; the clock-cut
+    // blocks are staged in shared memory when they fit in 96 KB (c1: 23 -> ? us)
+    {
+        const long long ks = K.tm_small.load();
+        const size_t ssmem = tm_finish_smem(nm, 1, n_f, a.xs, t.nslot) + (size_t)(F + 2) * 4 + 16;
+        size_t sblk = 0;
+        for (int m = 0; m < nm; ++m)
+            if (t.slot_of[m] >= 0) sblk += (size_t)dms[m]->nblk * 32;
+        const bool stage = sblk <= 96 * 1024 && ssmem + sblk <= (size_t)ds->small_dyn_max;
+        if (ks != 0 && n_k <= INT_MAX && ssmem <= (size_t)ds->small_dyn_max &&
+            (ks > 0 || (n_k <= ds->sms && (long long)tt * n_f <= 4096))) {
+            *launches = 0;
+            if (prepare_only) return ok();
+            a.tile_k = 1;
+            t.s = a;
+            t.slab0 = 0;
+            t.nks = (int)n_k;
+            const size_t sm = ssmem + (stage ? sblk : 0);
+            cudaError_t e;
+            {
+                KernelTimer ktm("k_tm_small", st);
+                const unsigned g = (unsigned)n_k;
+                switch ((fxall ? 1 : 0) + (stage ? 2 : 0)) {
+                    case 0: k_tm_small<false, false><<<g, 512, sm, st>>>(t); break;
+                    case 1: k_tm_small<true, false><<<g, 512, sm, st>>>(t); break;
+                    case 2: k_tm_small<false, true><<<g, 512, sm, st>>>(t); break;
+                    default: k_tm_small<true, true><<<g, 512, sm, st>>>(t); break;
+                }
+                e = cudaGetLastError();
+            }
+            if (e != cudaSuccess) return cuda_fail(e, "k_tm_small launch");
+            *launches = 1;
+            return ok();
+        }
+    }
     // large batches (>= 8 tasks per lane): 1024-thread CTAs and 1024-kernel feature blocks
     int NTW = tm_nt(std::min<long long>(n_k, 1LL << 40) * tt, ds->sms);
     if (tm_walk_smem(F, 32, tt, 0, NTW) > (size_t)ds->walk_dyn_max) NTW = 512;
@@ -590,7 +635,6 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
     }
     // finish tile: KT kernels per CTA, fp64 + fp32 per (model, kernel, clock) in shared memory
     // (small: the finish is a latency chain per CTA, so small batches want many CTAs)
-    a.xs = (F + 2) | 1;
     const int fnt = 256;
     auto fsmem_of = [&](int k) { return tm_finish_smem(nm, k, n_f, a.xs, t.nslot); };
     int kt_cap = 1;
@@ -1031,7 +1075,7 @@ syn_status run_sweep(const syn_model* const* models, int nm, const float* d_feat
     a.n_t = mode == kModeSweep && !prepare_only ? n_t : 0;
     for (int t = 0; t < a.n_t; ++t) {
         a.kind[t] = targets[t].kind;
-        a.x[t] = targets[t].x;
+        a.frac[t] = (double)targets[t].x / 100.0;   // the oracle's frac (oracle.c select)
     }
     a.choice = d_choice;
     a.S_out = pred[0];
@@ -1547,7 +1591,7 @@ syn_status synergy_select(const float* d_S, const float* d_E, int64_t n_k, int32
     a.n_t = n_t;
     for (int t = 0; t < n_t; ++t) {
         a.kind[t] = targets[t].kind;
-        a.x[t] = targets[t].x;
+        a.frac[t] = (double)targets[t].x / 100.0;   // the oracle's frac (oracle.c select)
     }
     a.choice = d_choice;
     int dev = 0;
@@ -1609,7 +1653,7 @@ syn_status synergy_choice_error(const float* d_S, const float* d_E, int64_t n_k,
     a.n_t = n_t;
     for (int t = 0; t < n_t; ++t) {
         a.kind[t] = targets[t].kind;
-        a.x[t] = targets[t].x;
+        a.frac[t] = (double)targets[t].x / 100.0;   // the oracle's frac (oracle.c select)
     }
     int dev = 0;
     cudaGetDevice(&dev);

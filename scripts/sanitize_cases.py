@@ -56,6 +56,12 @@ def main():
     run(W.make_config("c1"))
     syn.config_set("algo", 0)
     print("ok svr fp64 + general path", flush=True)
+    syn.config_set("tm_small", 0)                            # c1 on the two-kernel walk path too
+    run(W.make_config("c1"))
+    syn.config_set("tm_small", 1)                            # and the single-launch path on a fuzz case
+    run(W.fuzz_workload(1008, 40, 70, F=6, n_trees=5, max_depth=9, linear="both"))
+    syn.config_set("tm_small", -1)
+    print("ok walk / single-launch paths", flush=True)
     if mode == "full":
         syn.config_set("tm_slab", 64)
         syn.config_set("tm_kb", 32)
@@ -63,7 +69,13 @@ def main():
         run(w)
         print("ok slab pipeline", flush=True)
         syn.config_set("tm_slab", 0)
+        for kb in (512, 1024):                               # the large-batch block shapes
+            syn.config_set("tm_kb", kb)
+            syn.config_set("tm_nt", 1024)
+            run(W.make_config("c2"))
+            print("ok kb", kb, flush=True)
         syn.config_set("tm_kb", 0)
+        syn.config_set("tm_nt", 0)
         s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
         w = W.make_config("c1")
         with torch.cuda.stream(s1):

@@ -41,6 +41,7 @@ def _build():
 #             overlapping walk(i + 1), D double-buffered and re-zeroed by the finishes)
 #   tm_slab_seq  kernel slabs of 64 run in order on the caller's stream (one D buffer)
 VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 3},
+            "tm_small": {"tm_small": 1}, "tm_walk": {},
             "tm_kb32": {"tm_kb": 32}, "tm_ctas3": {"tm_ctas": 3},
             "tm_nsub3": {"tm_nsub": 3}, "tm_nsub64": {"tm_nsub": 64},
             "tm_dyn": {"tm_dyn": 1}, "tm_static": {"tm_dyn": 0}, "tm_nopdl": {"tm_pdl": 0},
@@ -48,8 +49,13 @@ VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 
             "tm_kb1024": {"tm_kb": 1024, "tm_nt": 1024},
             "tm_slab": {"tm_slab": 64, "tm_kb": 32},
             "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0}}
+# the walk variants ("tm_*" except tm_small) keep small batches on k_tm_walk + k_tm_finish too
+for _k, _v in VARIANTS.items():
+    if _k.startswith("tm_") and _k != "tm_small":
+        _v.setdefault("tm_small", 0)
 KNOB_DEFAULTS = {"algo": 0, "tm_kb": 0, "tm_ctas": 0, "tm_nsub": 0, "tm_split": -1, "tm_dyn": -1, "tm_pdl": 1,
-                 "tm_slab": 0, "tm_pipe": 1, "tm_kt": 0, "gen_kt": 0, "tm_nt": 0}
+                 "tm_slab": 0, "tm_pipe": 1, "tm_kt": 0, "gen_kt": 0, "tm_nt": 0,
+                 "tm_small": -1}
 
 
 def set_knobs(values):

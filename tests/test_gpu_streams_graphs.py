@@ -127,3 +127,28 @@ def test_unprepared_capture_is_refused():
             call()
     assert ei.value.status == syn.SYN_ERR_UNSUPPORTED
     torch.cuda.synchronize()
+
+
+def test_single_launch_path_prepare_then_capture():
+    """A small batch takes the single-launch k_tm_small (no difference arrays): prepare makes the
+    clock-cut copies, then the call is captured and replayed."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = W.fuzz_workload(10, 40, 64, F=5, n_trees=4, max_depth=8, p_leaf=0.1)
+    S, E, out = _buffers(w)
+    s = torch.cuda.Stream()
+    keep, call = _run(w, s.cuda_stream, S, E, out)
+    syn.prepare([keep[0], keep[1]], w.n_kernels, w.n_features, keep[2], stream=s.cuda_stream)
+    torch.cuda.synchronize()
+    with torch.cuda.stream(s):
+        call()
+    torch.cuda.synchronize()
+    assert syn.last_launch()["kernels"] == 1              # k_tm_small alone
+    S.fill_(-1.0); E.fill_(-1.0); out.fill_(-9)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        call()
+    for _ in range(2):
+        g.replay()
+    torch.cuda.synchronize()
+    _check(w, S, E, out)
