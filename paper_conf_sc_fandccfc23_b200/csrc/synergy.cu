@@ -734,12 +734,13 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
         }
         {
             KernelTimer ktm("k_tm_finish", fst);
+            const dim3 fgrid((unsigned)((t.nks + kt - 1) / kt));
             if (!pipe && K.tm_pdl.load() != 0) {
                 // programmatic dependent launch: the finish grid is scheduled while the walk runs
                 // and waits (griddepcontrol.wait) for it before reading D
                 cudaLaunchConfig_t lc;
                 memset(&lc, 0, sizeof lc);
-                lc.gridDim = dim3((unsigned)((t.nks + kt - 1) / kt));
+                lc.gridDim = fgrid;
                 lc.blockDim = dim3((unsigned)fnt);
                 lc.dynamicSmemBytes = fsmem;
                 lc.stream = fst;
@@ -750,7 +751,7 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
                 lc.numAttrs = 1;
                 e = cudaLaunchKernelEx(&lc, k_tm_finish, t);
             } else {
-                k_tm_finish<<<(unsigned)((t.nks + kt - 1) / kt), fnt, fsmem, fst>>>(t);
+                k_tm_finish<<<fgrid, fnt, fsmem, fst>>>(t);
                 e = cudaGetLastError();
             }
         }
