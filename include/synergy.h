@@ -269,11 +269,14 @@ syn_status synergy_last_launch(int32_t *kernels_launched, int64_t *evals, int64_
  * kernel launch is bracketed by two CUDA events recorded on its launch stream (two extra stream
  * operations per launch; off by default).  synergy_timing_read synchronises the recorded events,
  * sums the elapsed time per kernel name since the previous read, clears the record and returns
- * up to `cap` entries: names[k] (static strings, e.g. "k_sweep_da", "k_svr"), total_ms[k],
- * launches[k]; *n_kernels = number of distinct kernels recorded.  Process-wide, thread-safe. */
+ * up to `cap` entries: names[k] (static strings, e.g. "k_tm_walk", "k_svr_tc"), total_ms[k] (sum of
+ * the launch durations), busy_ms[k] (length of the union of the launch intervals, on the time axis
+ * of the first recorded event: less than total_ms when launches of one kernel overlap on several
+ * streams, as the slab pipeline's walks do; busy_ms may be NULL), launches[k]; *n_kernels = number
+ * of distinct kernels recorded.  Process-wide, thread-safe. */
 syn_status synergy_timing_enable(int32_t on);
-syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms, int64_t *launches,
-                               int32_t *n_kernels);
+syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms, double *busy_ms,
+                               int64_t *launches, int32_t *n_kernels);
 
 /* Tuning knobs (launch-configuration choices only; results are identical for every setting), for
  * tests and benchmarks.  Initialised once from the environment (SYNERGY_<KEY upper-case>), then
@@ -281,7 +284,9 @@ syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms
  * kernels per feature block, 32..1024), "tm_nt" (k_tm_walk threads per CTA, 512 or 1024), "tm_ctas",
  * "tm_nsub", "tm_split" (per-tree clock-range split, -1 automatic, 0 off, 1 on), "split_piece"
  * (model create: target cost of one split piece in quarters of the mean tree cost, default 4),
- * "tm_dyn" (task pools, -1 automatic), "tm_pdl" (default 1), "tm_slab", "tm_pipe" (default 1),
+ * "tm_dyn" (task pools, -1 automatic), "tm_pdl" (default 1), "tm_slab", "tm_pipe" (slab pipeline:
+ * 0 in order on the caller's stream, 1 finishes on a side stream, 2 (default) also the walks
+ * alternating between the caller's stream and a second walk stream),
  * "tm_kt", "gen_kt", "svr_splits", "svr_tc" (tcgen05 SVR contraction, default 1), "tm_small"
  * (single-launch k_tm_small for small batches: -1 automatic, 0 off, 1 on); 0 = automatic
  * unless noted.  INVALID_ARG: unknown key. */

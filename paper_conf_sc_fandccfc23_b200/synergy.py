@@ -84,7 +84,7 @@ def load(path: str = LIB_PATH) -> C.CDLL:
         "synergy_sweep_host": (I32, [P, P, P, P, I64, I32, P, I32, P, I32, P, P]),
         "synergy_last_launch": (I32, [P, P, P, P, P]),
         "synergy_timing_enable": (I32, [I32]),
-        "synergy_timing_read": (I32, [I32, P, P, P, P]),
+        "synergy_timing_read": (I32, [I32, P, P, P, P, P]),
         "synergy_prepare": (I32, [P, I32, I64, I32, P, P]),
         "synergy_config_set": (I32, [C.c_char_p, I64]),
         "synergy_config_get": (I32, [C.c_char_p, P]),
@@ -381,10 +381,12 @@ def timing_enable(on: bool = True):
 
 
 def timing_read(cap: int = 32):
-    """synergy_timing_read: {kernel name: (total_ms, launches)} since the previous read."""
+    """synergy_timing_read: {kernel name: (total_ms, launches, busy_ms)} since the previous read
+    (busy_ms: the union of the kernel's launch intervals)."""
     names = (C.c_char_p * cap)()
     ms = (C.c_double * cap)()
+    busy = (C.c_double * cap)()
     cnt = (C.c_int64 * cap)()
     n = C.c_int32()
-    _check(load().synergy_timing_read(cap, names, ms, cnt, C.byref(n)))
-    return {names[k].decode(): (ms[k], cnt[k]) for k in range(min(n.value, cap))}
+    _check(load().synergy_timing_read(cap, names, ms, busy, cnt, C.byref(n)))
+    return {names[k].decode(): (ms[k], cnt[k], busy[k]) for k in range(min(n.value, cap))}

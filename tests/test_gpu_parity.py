@@ -38,8 +38,10 @@ def _build():
 #   tm_kb1024 1024-thread CTAs with 1024-kernel feature blocks (the large-batch configuration)
 #   tm_nopdl  k_tm_finish launched without programmatic dependent launch
 #   tm_slab   kernel slabs of 64 (several walk + finish launches; finish(i) on the side stream
-#             overlapping walk(i + 1), D double-buffered and re-zeroed by the finishes)
+#             overlapping walk(i + 1), the walks alternating between two streams (tm_pipe 2,
+#             the default), D double-buffered and re-zeroed by the finishes)
 #   tm_slab_seq  kernel slabs of 64 run in order on the caller's stream (one D buffer)
+#   tm_slab1  kernel slabs of 64 with every walk on the caller's stream (tm_pipe 1)
 VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 3},
             "tm_small": {"tm_small": 1}, "tm_walk": {},
             "tm_kb32": {"tm_kb": 32}, "tm_ctas3": {"tm_ctas": 3},
@@ -48,13 +50,14 @@ VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 
             "tm_split": {"tm_split": 1}, "tm_nosplit": {"tm_split": 0}, "tm_nt1024": {"tm_nt": 1024},
             "tm_kb1024": {"tm_kb": 1024, "tm_nt": 1024},
             "tm_slab": {"tm_slab": 64, "tm_kb": 32},
-            "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0}}
+            "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0},
+            "tm_slab1": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 1}}
 # the walk variants ("tm_*" except tm_small) keep small batches on k_tm_walk + k_tm_finish too
 for _k, _v in VARIANTS.items():
     if _k.startswith("tm_") and _k != "tm_small":
         _v.setdefault("tm_small", 0)
 KNOB_DEFAULTS = {"algo": 0, "tm_kb": 0, "tm_ctas": 0, "tm_nsub": 0, "tm_split": -1, "tm_dyn": -1, "tm_pdl": 1,
-                 "tm_slab": 0, "tm_pipe": 1, "tm_kt": 0, "gen_kt": 0, "tm_nt": 0,
+                 "tm_slab": 0, "tm_pipe": 2, "tm_kt": 0, "gen_kt": 0, "tm_nt": 0,
                  "tm_small": -1}
 
 

@@ -152,3 +152,31 @@ def test_single_launch_path_prepare_then_capture():
         g.replay()
     torch.cuda.synchronize()
     _check(w, S, E, out)
+
+
+@pytest.mark.gpu
+def test_timing_busy_is_union_of_launch_intervals(slabs64):
+    """synergy_timing_read's busy time is the union of a kernel's launch intervals: never above the
+    summed launch durations, and below it only when launches overlap (the slab pipeline's walks on
+    two streams); results are unchanged with timing on."""
+    import torch
+    from paper_conf_sc_fandccfc23_b200 import synergy as syn
+    w = _workload(77)
+    S, E, out = _buffers(w)
+    _, fn = _run(w, None, S, E, out)
+    fn()
+    torch.cuda.synchronize()
+    syn.timing_read()
+    syn.timing_enable(True)
+    try:
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+    finally:
+        syn.timing_enable(False)
+    t = syn.timing_read()
+    assert "k_tm_walk" in t and "k_tm_finish" in t
+    for name, (total, launches, busy) in t.items():
+        assert launches > 0 and total > 0.0
+        assert 0.0 < busy <= total * (1 + 1e-6) + 1e-3, (name, total, busy)
+    _check(w, S, E, out)
