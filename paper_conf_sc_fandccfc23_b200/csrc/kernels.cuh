@@ -25,13 +25,20 @@ __device__ __forceinline__ bool valid_pred(float s, float e) {
 }
 
 // Model output from its forest sum (the exact leaf sum rounded once to fp64; oracle order: linear
-// member first, then the forest mean; a weight of exactly 1 skips its multiplication, Q7).
-__device__ __forceinline__ double combine(const DevModel& m, double forest_sum, const float* xrow, float f, int F) {
+// member first, then the forest mean; a weight of exactly 1 skips its multiplication, Q7).  The
+// linear member's fma chain runs over the F static inputs, then the clock (input F): its static
+// part is the same for every clock of a kernel, so linear_static() computes it once per (kernel,
+// model) and combine_pre() finishes each clock with the same operations in the same order.
+__device__ __forceinline__ double linear_static(const DevModel& m, const float* xrow, int F) {
+    double lin = m.lin_b;
+    if (m.lin_weight != 0.0)
+        for (int j = 0; j < F; ++j) lin = __fma_rn(__ldg(m.lin_w + j), (double)xrow[j], lin);
+    return lin;
+}
+__device__ __forceinline__ double combine_pre(const DevModel& m, double forest_sum, double lin_s, float f, int F) {
     double out = 0.0;
     if (m.lin_weight != 0.0) {
-        double lin = m.lin_b;
-        for (int j = 0; j < F; ++j) lin = __fma_rn(__ldg(m.lin_w + j), (double)xrow[j], lin);
-        lin = __fma_rn(__ldg(m.lin_w + F), (double)f, lin);
+        const double lin = __fma_rn(__ldg(m.lin_w + F), (double)f, lin_s);
         out = __dadd_rn(out, m.lin_weight == 1.0 ? lin : __dmul_rn(m.lin_weight, lin));
     }
     if (m.forest_weight != 0.0) {
@@ -39,6 +46,9 @@ __device__ __forceinline__ double combine(const DevModel& m, double forest_sum, 
         out = __dadd_rn(out, m.forest_weight == 1.0 ? forest : __dmul_rn(m.forest_weight, forest));
     }
     return out;
+}
+__device__ __forceinline__ double combine(const DevModel& m, double forest_sum, const float* xrow, float f, int F) {
+    return combine_pre(m, forest_sum, linear_static(m, xrow, F), f, F);
 }
 
 // Selection on integer keys.  A valid prediction (Q16) is a positive finite float, and the bit

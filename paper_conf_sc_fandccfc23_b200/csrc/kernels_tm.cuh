@@ -426,8 +426,9 @@ __device__ __forceinline__ void tm_finish_tile(const TmArgs& t, const TmFinishSm
         double* out = L.mv0 + ((size_t)pm * KT + pk) * n_f;
         const float* xrow = L.xk + pk * XS;
         const int slot = t.slot_of[pm];
+        const double lin_s = linear_static(m, xrow, F);                     // once per (kernel, model)
         if (slot < 0) {
-            for (int i = lane; i < n_f; i += 32) out[i] = combine(m, 0.0, xrow, L.fr[i], F);
+            for (int i = lane; i < n_f; i += 32) out[i] = combine_pre(m, 0.0, lin_s, L.fr[i], F);
             continue;
         }
         long long* Dm = L.sD + ((size_t)pk * t.nslot + slot) * n_f;
@@ -454,7 +455,7 @@ __device__ __forceinline__ void tm_finish_tile(const TmArgs& t, const TmFinishSm
 #pragma unroll 4
         for (int i = lane; i < n_f; i += 32) {
             const double forest_sum = __dmul_rn(__ll2double_rn(Dm[i]), inv);  // RN(exact sum)
-            out[i] = combine(m, forest_sum, xrow, L.fr[i], F);
+            out[i] = combine_pre(m, forest_sum, lin_s, L.fr[i], F);
         }
     }
     __syncthreads();
