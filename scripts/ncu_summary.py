@@ -1,6 +1,8 @@
 """Summarise ncu --set full reports (one kernel each) into a markdown table.
 
-    python scripts/ncu_summary.py OUT.md TITLE label1=report1.ncu-rep label2=report2.ncu-rep ...
+    python scripts/ncu_summary.py OUT.md TITLE label1=report1.ncu-rep label2=report2.ncu-rep#1 ...
+
+(`#i` picks the i-th kernel of a report that holds several; default the first.)
 """
 import csv
 import io
@@ -36,13 +38,25 @@ METRICS = [
     "launch__block_size",
     "launch__shared_mem_per_block_dynamic",
     "sm__cycles_elapsed.avg",
+    "sm__cycles_active.avg",
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_red.sum",
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_ld_lookup_miss.sum",
+    "smsp__average_warps_issue_stalled_branch_resolving_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_no_instruction_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio",
+    "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+    "sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active",
 ]
 
 
 def raw(rep):
+    idx = 0
+    if "#" in rep:
+        rep, idx = rep.rsplit("#", 1)
+        idx = int(idx)
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
-    h, u, v = rows[0], rows[1], rows[2]
+    h, u, v = rows[0], rows[1], rows[2 + idx]
     return v[h.index("Kernel Name")], {k: (v[h.index(k)], u[h.index(k)]) for k in METRICS if k in h}
 
 
