@@ -7,12 +7,15 @@
 // shared-memory limits checked by the host (tm_eligible); kernels_gen.cuh takes the rest.  The
 // work is laid on the machine to cut L1 wavefronts, the resource a kernel-major walk saturates:
 //
-//  * Tree-major lanes.  A lane task is one (kernel, model, tree).  Tasks are numbered
+//  * Tree-major lanes.  A lane task is one (kernel, model, tree) (or a clock sub-range of one,
+//    SUB).  Tasks are numbered
 //      j = ((kernel block) * TT + tree) * KB + kernel-in-block
 //    and every CTA owns a contiguous range of j, so the lanes of an SM walk the SAME few trees for
-//    up to KB different kernels at once: the SM's L1 holds those trees, the 32 lanes of a warp
-//    load blocks of one tree (shared lines), and lines are reused by every kernel of the block.
-//    (round 1's kernel-major k_sweep_da ran ~1000 different trees per SM: 9% L1 hits on c3.)
+//    up to KB different kernels at once: the SM's L1 holds those trees (block loads hit L1 ~97 %
+//    of the time on c3), the 32 lanes of a warp load blocks of one tree, and lines are reused by
+//    every kernel of the block.  Within a CTA, lane l of every warp takes the tasks j = l mod 32
+//    in order from its pool's shared counter (per-lane-index task pools), so short walks are
+//    balanced by taking the remaining tasks and a warp's kernels stay distinct mod 32.
 //
 //  * Resume walks.  For a fixed kernel a tree is a step function of the clock index.  walk(lo)
 //    follows clock lo's path; the run is [lo, hi) with hi = #{i : f_i <= thr} minimised over the
@@ -36,16 +39,17 @@
 //
 //  * Step-level lockstep.  Every loop iteration is one 2-level block step for every busy lane; a
 //    lane that reaches a leaf closes its run and resumes in the same iteration, so walks of
-//    different lengths do not idle lanes.  Each lane keeps its kernel's features in its own
-//    shared-memory column with the walked clock as row F, so every split reads x[code] with no
-//    clock/feature select, and clock splits and leaves are flagged in the block (k_cut_blocks).
+//    different lengths do not idle lanes.  The kernel block's static features sit once per
+//    segment in a transposed shared table [F + 2][KB] (kernel kk in bank kk mod 32 of every row),
+//    the walked clock is a register, and clock splits and leaves are flagged in the block
+//    (k_cut_blocks); a step reads the node's input, decides, then reads the taken child's.
 //
 //  * Accumulation in L2.  Run j of a (kernel, model, tree) adds v_j - v_{j-1} to
 //    D[kernel][slot][lo_j] with one 64-bit global reduction (exact, order-free; run 0 adds v_0).
-//    No shared-memory difference arrays: shared memory stays ~54 KB per CTA so L1 keeps the
-//    trees.  k_tm_finish then scans each D row (exact int64 prefix sum = the exact leaf sum per
-//    clock), rounds it once, combines the members and runs finish_tile4; it zeroes D as it reads
-//    it, so the next call starts from zeros without a memset.
+//    No shared-memory difference arrays (a slab's D rows are tens of MB).  k_tm_finish then scans
+//    each D row (exact int64 prefix sum = the exact leaf sum per clock), rounds it once, combines
+//    the members and runs finish_tile4; it zeroes D as it reads it, so the next call starts from
+//    zeros without a memset.
 #pragma once
 #include "kernels.cuh"
 
