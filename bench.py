@@ -515,7 +515,8 @@ def main():
         per_step = max(1.0, ktimes["k_svr_tc"][1] / K)
         n_k_l = evals_step // n_f
         n_svp = -(-en_spec.n_sv // 32) * 32
-        ops = 28 * 2.0 * (-(-n_k_l // 128) * 128) * (-(-n_f // 64) * 64) * n_svp / per_step
+        tc_n = 32                                           # kTcN: clocks per k_svr_tc tile (kernels_svr_tc.cuh)
+        ops = 28 * 2.0 * (-(-n_k_l // 128) * 128) * (-(-n_f // tc_n) * tc_n) * n_svp / per_step
         roofline["svr_contraction"] = {
             "bound": "tensor", "kernel": "k_svr_tc", "kernel_ms": tc_s * 1e3, "achieved": ops / tc_s / 1e12,
             "peak": 2.0 * peaks["bf16_tflops"], "unit": "TOP/s (int8)",

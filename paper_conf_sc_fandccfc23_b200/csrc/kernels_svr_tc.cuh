@@ -13,7 +13,7 @@
 //   * U V = 2^(eU + 1 - 108) sum_{p,q} 256^(12-p-q) (D_p E_q), and each digit product D_p E_q is an
 //     int8 x int8 GEMM with exact int32 accumulation (tcgen05.mma kind::i8; |sum| <= 128^2 * n_sv
 //     * 7 < 2^31 for n_sv <= 16384).  Products of equal level L = p + q share one TMEM accumulator
-//     (7 levels x 64 columns); levels L >= 7 are dropped (the 28 pairs with L <= 6 are kept);
+//     (7 levels x 32 columns); levels L >= 7 are dropped (the 28 pairs with L <= 6 are kept);
 //   * the epilogue reads the 7 level accumulators (tcgen05.ld), sums 2^-(8L+12) acc_L in fp64 and
 //     scales by 2^(eU + 1).  Digit rounding and the dropped levels change each term by at most
 //     about 2^-53 max_j|dual_j| (both factors' scales are powers of two), so the value is within
@@ -25,9 +25,12 @@
 // canonical K-major, no-swizzle UMMA layout (8-row x 16-byte core matrices; LBO = 128 B between the
 // two K-adjacent core matrices of a 32-SV chunk, SBO = 256 B between 8-row groups), all 8 digit
 // planes of a (tile, chunk) contiguous, so each chunk reaches shared memory by one 1-D bulk copy per
-// operand (cp.async.bulk, the TMA engine) into a 4-stage mbarrier ring.  k_svr_tc: 128 kernels x 64
-// clocks per CTA (M = 128, N = 64, K = 32 per MMA); warp 0 producer, warp 1 TMEM allocation and
-// MMA issue (one elected lane, 28 MMAs per chunk), warps 2-5 epilogue (TMEM lane quarters).  The SV
+// operand (cp.async.bulk, the TMA engine) into a 3-stage mbarrier ring.  k_svr_tc: 128 kernels x 32
+// clocks per CTA (M = 128, N = 32, K = 32 per MMA), two CTAs per SM (105 KB of shared memory and
+// 256 TMEM columns each), so one CTA's MMAs overlap the other's epilogue and operand loads (the
+// N = 64, one-CTA-per-SM version took 0.36 ms per c3 slab, this one 0.30); warp 0 producer, warp
+// 1 TMEM allocation and MMA issue (one elected lane, 28 MMAs per chunk), warps 2-5 epilogue (TMEM
+// lane quarters).  The SV
 // range may be split across CTAs (blockIdx.z); each split writes its partial plane P[z], which the
 // finish sums in split order (add_svr_unit), exactly as for k_svr.
 #pragma once
@@ -35,17 +38,18 @@
 
 namespace syn {
 
-constexpr int kTcM = 128, kTcN = 64, kTcKC = 32, kTcDig = 7, kTcStages = 4;
+constexpr int kTcM = 128, kTcN = 32, kTcKC = 32, kTcDig = 7, kTcStages = 3;
 constexpr unsigned kTcAPlane = (unsigned)kTcM * kTcKC, kTcBPlane = (unsigned)kTcN * kTcKC;
 constexpr unsigned kTcABytes = kTcDig * kTcAPlane;   // one 32-SV chunk of U, all digit planes
 constexpr unsigned kTcBBytes = kTcDig * kTcBPlane;   // one chunk of V
 constexpr int kTcThreads = 192;
+constexpr int kTcCtasPerSm = 2;                      // 3-stage ring (105 KB) and 256 TMEM columns each
 constexpr size_t kTcSmem = (size_t)kTcStages * (kTcABytes + kTcBBytes) + 256;
 
 struct SvrTcArgs {
     SvrArgs s;               // features, clocks, SVs, duals, standardisation, gamma, slab
     unsigned char* Uq;       // [mtiles of the slab][n_chunks][kTcDig][128 x 32] int8
-    unsigned char* Vq;       // [ntiles][n_chunks][kTcDig][64 x 32] int8
+    unsigned char* Vq;       // [ntiles][n_chunks][kTcDig][kTcN x 32] int8
     int eU;                  // U scale exponent (max |dual| < 2^eU)
     int chunks_per_split;
 };
@@ -120,7 +124,7 @@ __global__ void __launch_bounds__(256) k_svr_udig(const __grid_constant__ SvrTcA
     tc_store_digits(x, t.Uq + ((size_t)mt * n_chunks + c) * kTcABytes + tc_off(r, 16 * h), kTcAPlane);
 }
 
-// V digits for a 64-clock tile (blockIdx.x) and a 32-SV chunk (blockIdx.y): thread = (clock r,
+// V digits for a kTcN-clock tile (blockIdx.x) and a 32-SV chunk (blockIdx.y): thread = (clock r,
 // 16-SV half h).  V_ji = exp(-gamma (z(f_i) - sv_jF)^2) (k_svr_v's arithmetic), scaled by 2^-1.
 __global__ void __launch_bounds__(128) k_svr_vdig(const __grid_constant__ SvrTcArgs t) {
     const SvrArgs& a = t.s;
@@ -150,11 +154,11 @@ __device__ __forceinline__ unsigned long long tc_desc(unsigned saddr) {
 }
 
 // tcgen05.mma kind::i8 instruction descriptor: s32 accumulator, signed int8 A and B, both K-major,
-// M = 128, N = 64.
+// M = 128, N = kTcN.
 constexpr unsigned kTcIdesc = (2u << 4) | (1u << 7) | (1u << 10) | ((unsigned)(kTcN >> 3) << 17) |
                               ((unsigned)(kTcM >> 4) << 24);
 
-__global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant__ SvrTcArgs t) {
+__global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm) k_svr_tc(const __grid_constant__ SvrTcArgs t) {
     const SvrArgs& a = t.s;
     extern __shared__ __align__(128) unsigned char tcs[];
     unsigned char* As = tcs;                                             // [stages][A chunk]
@@ -178,8 +182,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant_
         mbar_init(accb, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (warp == 1) {                                                     // 512 TMEM columns: 7 x 64 used
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;"
+    if (warp == 1) {                                                     // 256 TMEM columns: 7 x 32 used
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;"
                      :: "r"(svr_su32(tmem_slot)) : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     }
@@ -270,7 +274,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_svr_tc(const __grid_constant_
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
     if (warp == 1)
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" :: "r"(tmem) : "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 256;" :: "r"(tmem) : "memory");
 }
 
 }  // namespace syn

@@ -866,7 +866,8 @@ syn_status prepare_svr_tc(DevModel& dm, DevState* ds, const float* d_features, l
     long long nks = std::max<long long>(kTcM, (long long)(kSvrSlabBytes / ((size_t)n_svp * kTcDig)) / kTcM * kTcM);
     nks = std::min<long long>(nks, (n_k + kTcM - 1) / kTcM * kTcM);
     const long long tiles = (std::min(nks, n_k) + kTcM - 1) / kTcM * tiles_n;
-    int splits = (int)std::max<long long>(1, ds->sms / std::max<long long>(tiles, 1));
+    // split the SV range until the grid covers the resident CTA slots (kTcCtasPerSm per SM)
+    int splits = (int)std::max<long long>(1, (long long)kTcCtasPerSm * ds->sms / std::max<long long>(tiles, 1));
     splits = std::min(splits, kSvrMaxSplits);
     if (knobs().svr_splits.load() > 0) splits = (int)std::min<long long>(knobs().svr_splits.load(), kSvrMaxSplits);
     splits = std::max(1, std::min(splits, n_chunks));
