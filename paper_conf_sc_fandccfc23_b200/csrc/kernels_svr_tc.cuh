@@ -61,27 +61,35 @@ __device__ __forceinline__ unsigned tc_off(int r, int kb) {
 }
 
 // 16 consecutive values (x[q] in (-1, 1)) -> kTcDig digit planes, 16 bytes each, at base + p * plane.
-// X = round(x 2^54) (an integer, |X| < 2^54) is written in balanced base 256, least significant
-// digit first: d = ((X + 128) mod 256) - 128 in [-128, 127], X = (X - d) / 256 (exact), so
-// X = sum_p d_p 256^(kTcDig - 1 - p) with every digit a signed byte; |x - X 2^-54| <= 2^-55.
+// X = round(x 2^54) (an integer, |X| <= 2^54) is written in balanced base 256: the unique digits
+// d_p in [-128, 127] with X = sum_p d_p 256^(kTcDig - 1 - p); |x - X 2^-54| <= 2^-55.  With
+// C = 0x0080808080808080 (128 in each of the 7 digit positions), X + C is in [0, 256^7) and its
+// base-256 digits are d_p + 128, so the signed bytes of (X + C) xor C are exactly the d_p (the
+// digit-by-digit recurrence d = ((X + 128) mod 256) - 128, X = (X - d) / 256 gives the same digits).
 __device__ __forceinline__ void tc_store_digits(const double (&x)[16], unsigned char* base, unsigned plane) {
-    long long X[16];
+    constexpr unsigned long long C = 0x0080808080808080ull;
+    unsigned lo[16], hi[16];
 #pragma unroll
-    for (int q = 0; q < 16; ++q) X[q] = __double2ll_rn(scalbn(x[q], 54));
-    unsigned w[kTcDig][4];
-#pragma unroll
-    for (int p = kTcDig - 1; p >= 0; --p) {
-        w[p][0] = w[p][1] = w[p][2] = w[p][3] = 0u;
-#pragma unroll
-        for (int q = 0; q < 16; ++q) {
-            const long long d = ((X[q] + 128) & 255) - 128;
-            X[q] = (X[q] - d) >> 8;                                        // exact
-            w[p][q >> 2] |= ((unsigned)d & 0xffu) << (8 * (q & 3));
-        }
+    for (int q = 0; q < 16; ++q) {
+        const unsigned long long Z = ((unsigned long long)__double2ll_rn(scalbn(x[q], 54)) + C) ^ C;
+        lo[q] = (unsigned)Z;
+        hi[q] = (unsigned)(Z >> 32);
     }
 #pragma unroll
-    for (int p = 0; p < kTcDig; ++p)
-        *reinterpret_cast<uint4*>(base + (size_t)p * plane) = make_uint4(w[p][0], w[p][1], w[p][2], w[p][3]);
+    for (int p = 0; p < kTcDig; ++p) {
+        const int bi = kTcDig - 1 - p;                                    // byte of Z holding d_p
+        unsigned w[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            const unsigned* h = bi < 4 ? lo : hi;
+            const unsigned j = (unsigned)(bi & 3);
+            const unsigned sel = j | ((4u + j) << 4);                    // [a_j, b_j] in bytes 0, 1
+            const unsigned t1 = __byte_perm(h[4 * k], h[4 * k + 1], sel);
+            const unsigned t2 = __byte_perm(h[4 * k + 2], h[4 * k + 3], sel);
+            w[k] = __byte_perm(t1, t2, 0x5410u);                          // values 4k .. 4k+3
+        }
+        *reinterpret_cast<uint4*>(base + (size_t)p * plane) = make_uint4(w[0], w[1], w[2], w[3]);
+    }
 }
 
 // U digits for a 128-kernel tile (blockIdx.x, slab-relative) and a 32-SV chunk (blockIdx.y):
