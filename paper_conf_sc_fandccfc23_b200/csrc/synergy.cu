@@ -1800,20 +1800,31 @@ syn_status synergy_timing_read(int32_t cap, const char** names, double* total_ms
     std::vector<std::vector<std::pair<double, double>>> iv;       // per kernel: launch intervals
     syn_status st = SYN_OK;
     const cudaEvent_t ref = g_tl.empty() ? nullptr : g_tl.front().a;
+    double far = 0.0;                                            // incomparable launches (see below)
     for (const TimedLaunch& t : g_tl) {
         float x = 0.0f, xa = 0.0f, xb = 0.0f;
         cudaError_t e = cudaEventSynchronize(t.b);
         if (e == cudaSuccess) e = cudaEventSynchronize(t.a);
         if (e == cudaSuccess) e = cudaEventElapsedTime(&x, t.a, t.b);
-        if (e == cudaSuccess) e = cudaEventElapsedTime(&xa, ref, t.a);    // on a common time axis
-        if (e == cudaSuccess) e = cudaEventElapsedTime(&xb, ref, t.b);
         if (e != cudaSuccess && st == SYN_OK) st = cuda_fail(e, "timing events");
+        // on a common time axis (the first event's); events of another device cannot be compared:
+        // such a launch counts as an interval of its own, placed after everything else
+        double ia, ib;
+        if (cudaEventElapsedTime(&xa, ref, t.a) == cudaSuccess && cudaEventElapsedTime(&xb, ref, t.b) == cudaSuccess) {
+            ia = xa;
+            ib = xb;
+        } else {
+            cudaGetLastError();
+            ia = 1e9 + far;
+            ib = ia + x;
+            far += (double)x + 1.0;
+        }
         size_t k = 0;
         while (k < nm.size() && strcmp(nm[k], t.name)) ++k;
         if (k == nm.size()) { nm.push_back(t.name); ms.push_back(0.0); cnt.push_back(0); iv.emplace_back(); }
         ms[k] += x;
         cnt[k] += 1;
-        iv[k].push_back({xa, xb});
+        iv[k].push_back({ia, ib});
     }
     for (const TimedLaunch& t : g_tl) {
         g_evpool.push_back(t.a);
