@@ -34,6 +34,8 @@ struct DevModel {
     // a root-to-leaf walk of depth D takes max(1, ceil(D / 2)) block loads.
     const uint4* blocks;
     const int* broot;        // [n_trees] root block of each tree
+    const int* broot_lpt;    // [n_trees] the same roots in expected-cost order, alternating the
+                             // costliest and the cheapest remaining tree (small batches, see run_tm)
     // per-tree clock sub-range split for small batches (k_tm_walk unit tables): {first unit of the
     // tree within the model, sub-ranges}; sub-ranges ~ ceil(expected runs / the model's mean), so
     // the longest (kernel, tree) walks are cut into pieces of about average length

@@ -81,6 +81,8 @@ struct TmArgs {
     int smode;                   // units: 0 one per tree, 1 nsub per tree, 2 per-tree split (tsplit)
     int units;                   // units per kernel block (tasks per kernel)
     int dyn;                     // k_tm_walk: tasks from a shared counter
+    int lpt;                     // the models' roots are in expected-cost order (broot_lpt): tree
+                                 // ranges are not contiguous in the blocks, so the prefetch differs
 };
 
 // One 2-level block step on clock-cut words (A = {thr(n), thr(c0), thr(c1), codes}, grandchild
@@ -124,7 +126,9 @@ struct __align__(16) TmTree {
 // SUB: a task is (kernel, unit) with a unit = (tree, clock sub-range [lo, end)) from a unit table
 // in shared memory (t.smode 1: every tree in t.nsub equal sub-ranges, tiny batches; 2: each tree
 // in its tsplit sub-ranges, small batches); otherwise a unit is a whole tree.
-template <int NT, bool FXALL, bool SUB>
+// LPT: the models' roots are the expected-cost order (broot_lpt, t.lpt): a compile-time variant so
+// that the other launches keep their code unchanged.
+template <int NT, bool FXALL, bool SUB, bool LPT = false>
 __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant__ TmArgs t) {
     const SweepArgs& a = t.s;
     extern __shared__ __align__(16) unsigned char smem[];
@@ -209,7 +213,23 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_tm_walk(const __grid_constant
         // pull the blocks of the segment's first trees (at most 8) into L2 with bulk prefetches
         // (one per model's contiguous tree range), so the first walks of a cold model do not
         // serialise DRAM misses; later trees of a long range arrive while the first are walked
-        if (threadIdx.x == 0) {
+        if (LPT && threadIdx.x == 0) {
+            // cost-ordered roots: CTA c pulls its share of every model's blocks instead (together
+            // the CTAs prefetch each model once)
+            for (int mi = 0; mi < 4; ++mi) {
+                if (!(mi == 0 ? T0 : mi == 1 ? T1 : mi == 2 ? T2 : T3)) continue;
+                const long long nb = s_nblk[mi];
+                const long long b0 = nb * blockIdx.x / gridDim.x, b1 = nb * (blockIdx.x + 1) / gridDim.x;
+                const char* p = reinterpret_cast<const char*>(model_of(a, mi).blocks + 2 * (size_t)b0);
+                size_t left = (size_t)(b1 - b0) * 32;
+                while (left > 0) {
+                    const unsigned n = (unsigned)min(left, (size_t)1 << 20);
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(n) : "memory");
+                    p += n;
+                    left -= n;
+                }
+            }
+        } else if (!LPT && threadIdx.x == 0) {
             const int ta = SUB ? units[seg0 >> KBL].x : seg0 >> KBL;
             const int tb = min(ta + 7, SUB ? units[(seg1 - 1) >> KBL].x : (seg1 - 1) >> KBL);
             int u = ta;

@@ -180,6 +180,7 @@ struct Knobs {
     std::atomic<long long> tm_dyn{-1};    // dynamic task fetch: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pdl{1};     // programmatic dependent launch of k_tm_finish
     std::atomic<long long> tm_slab{0};    // kernels per slab (0: D of one slab <= 48 MB)
+    std::atomic<long long> tm_lpt{-1};    // expected-cost tree order for ~1 task per lane: -1 auto, 0 off, 1 on
     std::atomic<long long> tm_pipe{2};    // slab pipeline: 1 finish on a side stream, 2 + two walk streams
     std::atomic<long long> tm_kt{0};      // k_tm_finish kernels per CTA
     std::atomic<long long> gen_kt{0};     // k_gen_finish kernels per CTA
@@ -194,7 +195,7 @@ struct KnobName {
 };
 const KnobName kKnobs[] = {{"algo", &g_knobs.algo},       {"tm_kb", &g_knobs.tm_kb},   {"tm_ctas", &g_knobs.tm_ctas},
                            {"tm_nsub", &g_knobs.tm_nsub}, {"tm_split", &g_knobs.tm_split}, {"tm_nt", &g_knobs.tm_nt}, {"split_piece", &g_knobs.split_piece}, {"tm_dyn", &g_knobs.tm_dyn}, {"tm_pdl", &g_knobs.tm_pdl},
-                           {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_kt", &g_knobs.tm_kt},
+                           {"tm_slab", &g_knobs.tm_slab}, {"tm_pipe", &g_knobs.tm_pipe}, {"tm_lpt", &g_knobs.tm_lpt}, {"tm_kt", &g_knobs.tm_kt},
                            {"gen_kt", &g_knobs.gen_kt}, {"svr_splits", &g_knobs.svr_splits},
                            {"svr_tc", &g_knobs.svr_tc}, {"tm_small", &g_knobs.tm_small}};
 std::once_flag g_knobs_once;
@@ -256,6 +257,8 @@ DevState* dev_state(int dev) {
         chk(allow_smem(k_tm_walk<1024, false, false>, d.optin));
         chk(allow_smem(k_tm_walk<1024, true, true>, d.optin));
         chk(allow_smem(k_tm_walk<1024, false, true>, d.optin));
+        chk(allow_smem(k_tm_walk<512, true, false, true>, d.optin));
+        chk(allow_smem(k_tm_walk<512, false, false, true>, d.optin));
         chk(allow_smem(k_tm_finish, d.optin));
         chk(allow_smem(k_tm_small<true, false>, d.optin));
         chk(allow_smem(k_tm_small<false, false>, d.optin));
@@ -719,6 +722,18 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             t.units = usplit;
         }
         t.n_tasks = (long long)((t.nks + kb - 1) / kb) * t.units * kb;
+        // about one task per lane (c2): the trees in expected-cost order, alternating the costliest
+        // and the cheapest remaining (broot_lpt), so each CTA's range starts with a costly tree and
+        // the lanes that finish first take the cheap ones (measured c2 walk 70 -> 66.5 us; with
+        // more tasks per lane the order cost c5 11 % and c3 2 %, so it stays off there)
+        {
+            const long long kl = K.tm_lpt.load();
+            t.lpt = (t.smode == 0 && NTW == 512 && (kl > 0 || (kl < 0 && !pipe && per_lane < 2 && (long long)t.nks * tt >= lanes)))
+                        ? 1 : 0;
+            DevModel* tm[4] = {&t.s.ms, &t.s.me, &t.s.mx[0], &t.s.mx[1]};
+            for (int m = 0; m < nm; ++m)
+                if (t.slot_of[m] >= 0) tm[m]->broot = t.lpt ? dms[m]->broot_lpt : dms[m]->broot;
+        }
         const size_t wsmem = tm_walk_smem(F, kb, tt, t.smode ? t.units : 0, NTW);
         // a few tasks per lane: dynamic task fetch balances walks of different lengths
         // per-lane-index task pools by default (L1-resident tree window, balanced, conflict-free);
@@ -729,8 +744,12 @@ syn_status run_tm(SweepArgs a, int nm, syn_model* const* models, const syn_clock
             KernelTimer ktm("k_tm_walk", wst);
             const int cls = (fxall ? 1 : 0) + (t.smode ? 2 : 0) + (NTW == 1024 ? 4 : 0);
             switch (cls) {
-                case 0: k_tm_walk<512, false, false><<<(unsigned)g, 512, wsmem, wst>>>(t); break;
-                case 1: k_tm_walk<512, true, false><<<(unsigned)g, 512, wsmem, wst>>>(t); break;
+                case 0: if (t.lpt) k_tm_walk<512, false, false, true><<<(unsigned)g, 512, wsmem, wst>>>(t);
+                        else k_tm_walk<512, false, false><<<(unsigned)g, 512, wsmem, wst>>>(t);
+                        break;
+                case 1: if (t.lpt) k_tm_walk<512, true, false, true><<<(unsigned)g, 512, wsmem, wst>>>(t);
+                        else k_tm_walk<512, true, false><<<(unsigned)g, 512, wsmem, wst>>>(t);
+                        break;
                 case 2: k_tm_walk<512, false, true><<<(unsigned)g, 512, wsmem, wst>>>(t); break;
                 case 3: k_tm_walk<512, true, true><<<(unsigned)g, 512, wsmem, wst>>>(t); break;
                 case 4: k_tm_walk<1024, false, false><<<(unsigned)g, 1024, wsmem, wst>>>(t); break;
@@ -1276,6 +1295,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     // whose clock interval (from the clock-split thresholds on the path) is not empty.  A tree gets
     // ceil(runs / the model's mean runs) sub-ranges, at most 8.
     std::vector<int2> tsplit;
+    std::vector<int> lpt;                                  // expected-cost order (broot_lpt)
     int units_split = 0;
     if (d->forest_weight != 0.0) {
         std::vector<double> cost((size_t)d->n_trees, 0.0);
@@ -1305,6 +1325,11 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
             mean += cost[t];
         }
         mean /= d->n_trees;
+        std::vector<int> by(d->n_trees);
+        for (int t = 0; t < d->n_trees; ++t) by[t] = t;
+        std::stable_sort(by.begin(), by.end(), [&](int x, int y) { return cost[x] > cost[y]; });
+        lpt.resize(d->n_trees);
+        for (int i = 0, lo = 0, hi = d->n_trees - 1; lo <= hi; ++i) lpt[i] = (i & 1) ? by[hi--] : by[lo++];
         tsplit.resize(d->n_trees);
         for (int t = 0; t < d->n_trees; ++t) {
             const double piece = mean * (double)std::max<long long>(1, knobs().split_piece.load()) / 4.0;
@@ -1395,7 +1420,10 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     const size_t off_mn = off_dc + (dcb + 255) / 256 * 256, off_sc = off_mn + (lb + 255) / 256 * 256;
     const size_t off_ts = ((has_svr ? off_sc + lb : off_r + rb) + 255) / 256 * 256;
     const size_t tsb = std::max<size_t>(tsplit.size(), 1) * sizeof(int2);
-    const size_t total = off_ts + tsb;
+    const size_t off_lp = (off_ts + tsb + 255) / 256 * 256;
+    std::vector<int> broot_lpt(lpt.size());
+    for (size_t i = 0; i < lpt.size(); ++i) broot_lpt[i] = broot[lpt[i]];
+    const size_t total = off_lp + rb;
     void* mem = nullptr;
     cudaError_t e = cudaMalloc(&mem, total);
     if (e != cudaSuccess) return cuda_fail(e, "cudaMalloc(model)");
@@ -1408,6 +1436,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
         (!blocks.empty() && (e = cudaMemcpy(base + off_b, blocks.data(), blocks.size() * sizeof(uint4), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (!broot.empty() && (e = cudaMemcpy(base + off_r, broot.data(), broot.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (!tsplit.empty() && (e = cudaMemcpy(base + off_ts, tsplit.data(), tsplit.size() * sizeof(int2), cudaMemcpyHostToDevice)) != cudaSuccess) ||
+        (!broot_lpt.empty() && (e = cudaMemcpy(base + off_lp, broot_lpt.data(), broot_lpt.size() * sizeof(int), cudaMemcpyHostToDevice)) != cudaSuccess) ||
         (has_svr && ((e = cudaMemcpy(base + off_sv, d->sv, svb, cudaMemcpyHostToDevice)) != cudaSuccess ||
                      (e = cudaMemcpy(base + off_dc, d->dual_coef, dcb, cudaMemcpyHostToDevice)) != cudaSuccess ||
                      (e = cudaMemcpy(base + off_mn, d->in_mean, lb, cudaMemcpyHostToDevice)) != cudaSuccess ||
@@ -1438,6 +1467,7 @@ syn_status synergy_model_create(const syn_model_desc* d, int32_t device, syn_mod
     m->dm.depth = max_depth;
     m->dm.blocks = reinterpret_cast<const uint4*>(base + off_b);
     m->dm.broot = reinterpret_cast<const int*>(base + off_r);
+    m->dm.broot_lpt = reinterpret_cast<const int*>(base + off_lp);
     m->dm.tsplit = reinterpret_cast<const int2*>(base + off_ts);
     m->dm.units_split = units_split;
     m->n_blocks = (long long)(blocks.size() >> 1);

@@ -42,6 +42,8 @@ def _build():
 #             the default), D double-buffered and re-zeroed by the finishes)
 #   tm_slab_seq  kernel slabs of 64 run in order on the caller's stream (one D buffer)
 #   tm_slab1  kernel slabs of 64 with every walk on the caller's stream (tm_pipe 1)
+#   tm_lpt    trees walked in expected-cost order (broot_lpt) forced on (automatic at ~1 task per lane)
+#   tm_nolpt  expected-cost order off
 VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 3},
             "tm_small": {"tm_small": 1}, "tm_walk": {},
             "tm_kb32": {"tm_kb": 32}, "tm_ctas3": {"tm_ctas": 3},
@@ -51,14 +53,15 @@ VARIANTS = {"default": {}, "gen": {"algo": 1}, "gen_kt3": {"algo": 1, "gen_kt": 
             "tm_kb1024": {"tm_kb": 1024, "tm_nt": 1024},
             "tm_slab": {"tm_slab": 64, "tm_kb": 32},
             "tm_slab_seq": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 0},
-            "tm_slab1": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 1}}
+            "tm_slab1": {"tm_slab": 64, "tm_kb": 32, "tm_pipe": 1},
+            "tm_lpt": {"tm_lpt": 1}, "tm_nolpt": {"tm_lpt": 0}}
 # the walk variants ("tm_*" except tm_small) keep small batches on k_tm_walk + k_tm_finish too
 for _k, _v in VARIANTS.items():
     if _k.startswith("tm_") and _k != "tm_small":
         _v.setdefault("tm_small", 0)
 KNOB_DEFAULTS = {"algo": 0, "tm_kb": 0, "tm_ctas": 0, "tm_nsub": 0, "tm_split": -1, "tm_dyn": -1, "tm_pdl": 1,
                  "tm_slab": 0, "tm_pipe": 2, "tm_kt": 0, "gen_kt": 0, "tm_nt": 0,
-                 "tm_small": -1}
+                 "tm_small": -1, "tm_lpt": -1}
 
 
 def set_knobs(values):
