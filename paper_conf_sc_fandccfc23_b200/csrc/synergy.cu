@@ -388,8 +388,10 @@ syn_status tm_buffer(DevState* ds, int dev, cudaStream_t st, size_t bytes, TmBuf
 }
 
 // Slab pipeline (several kernel slabs per call): the finish of slab i runs on a library-owned
-// second stream while the walk of slab i + 1 runs on the caller's stream, with D double-buffered.
-// One side stream and four events per (device, caller stream).
+// side stream while the walk of slab i + 1 runs (on the caller's stream, or with tm_pipe 2 on the
+// caller's stream for even slabs and a second library stream for odd ones), D double-buffered.
+// Two library streams (finishes; odd slabs' walks with tm_pipe 2) and six events per (device,
+// caller stream).
 struct TmAux {
     int dev;
     cudaStream_t st;
