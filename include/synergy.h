@@ -284,7 +284,8 @@ syn_status synergy_timing_read(int32_t cap, const char **names, double *total_ms
  * kernels per feature block, 32..1024), "tm_nt" (k_tm_walk threads per CTA, 512 or 1024), "tm_ctas",
  * "tm_nsub", "tm_split" (per-tree clock-range split, -1 automatic, 0 off, 1 on), "split_piece"
  * (model create: target cost of one split piece in quarters of the mean tree cost, default 4),
- * "tm_dyn" (task pools, -1 automatic), "tm_pdl" (default 1), "tm_slab", "tm_pipe" (slab pipeline:
+ * "tm_dyn" (task pools, -1 automatic), "tm_pdl" (default 1), "tm_slab", "tm_lpt" (expected-cost tree order for
+ * batches of about one task per lane: -1 automatic, 0 off, 1 on), "tm_pipe" (slab pipeline:
  * 0 in order on the caller's stream, 1 finishes on a side stream, 2 (default) also the walks
  * alternating between the caller's stream and a second walk stream),
  * "tm_kt", "gen_kt", "svr_splits", "svr_tc" (tcgen05 SVR contraction, default 1), "tm_small"
